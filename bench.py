@@ -1,0 +1,381 @@
+#!/usr/bin/env python
+"""Benchmark of LiteForm's hot path on B200 (one JSON line on rank 0).
+
+A STEP is one pass of the whole hot path over the
+workload: GPU configure statistics + eq. 7 / Algorithm 3 (lf_cell_configure),
+GPU CSR->CELL conversion (lf_cell_build), CELL SpMM with the C update
+(lf_spmm); for N > 1 each rank runs it on its row shard and C is
+all-gathered over NCCL.  metric = GFLOP/s = 2*nnz*J / t_step (whole job).
+
+    python bench.py [--gpus N --steps K --warmup W --config c2_rmat20]
+    python bench.py --impl reference     # the CPU oracle, same metric
+
+Workload: BASELINE.json configs[1] (R-MAT scale 20, edge factor 16, J = 128),
+synthetic, seeded (gen/).  Inputs are larger than L2 (B 512 MB, C 512 MB).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import gen  # noqa: E402
+
+METRIC = "SpMM GFLOP/s (2*nnz*J/t) and HBM GB/s vs ~8 TB/s at 1/2/4/8 B200"
+
+
+def peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            p = json.load(f)
+        return float(p["hbm_gbs"]), "measured"
+    except Exception:
+        return 6650.0, "fallback"
+
+
+def algorithmic_bytes(A_h, J):
+    """bytes_alg = nnz*(4+4) + U*J*4 + I*J*4: index + value of
+    every nonzero once, each needed B row once, every C row written once."""
+    U = int(np.count_nonzero(np.bincount(A_h.col_ind, minlength=A_h.n_cols))) if A_h.nnz else 0
+    return 8 * A_h.nnz + 4 * U * J + 4 * A_h.n_rows * J, U
+
+
+class ClockSampler:
+    """NVML sampling of SM clocks and throttle reasons during the timed region."""
+    REASONS = {0x4: "sw_power_cap", 0x8: "hw_slowdown", 0x20: "sw_thermal_slowdown", 0x40: "hw_thermal_slowdown",
+               0x80: "hw_power_brake_slowdown", 0x2: "applications_clocks_setting"}
+
+    def __init__(self, dev_index: int):
+        self.samples, self.reasons, self.ok = [], 0, False
+        try:
+            import pynvml
+            import torch
+            pynvml.nvmlInit()
+            uuid = str(torch.cuda.get_device_properties(dev_index).uuid)
+            try:
+                self.h = pynvml.nvmlDeviceGetHandleByUUID(uuid if uuid.startswith("GPU-") else "GPU-" + uuid)
+            except Exception:
+                self.h = pynvml.nvmlDeviceGetHandleByIndex(dev_index)
+            self.max_mhz = pynvml.nvmlDeviceGetMaxClockInfo(self.h, pynvml.NVML_CLOCK_SM)
+            self.nv = pynvml
+            self.ok = True
+        except Exception as e:  # pragma: no cover
+            self.err = str(e)
+        self._stop = threading.Event()
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                self.samples.append(self.nv.nvmlDeviceGetClockInfo(self.h, self.nv.NVML_CLOCK_SM))
+                self.reasons |= int(self.nv.nvmlDeviceGetCurrentClocksEventReasons(self.h))
+            except Exception:
+                pass
+            self._stop.wait(0.01)
+
+    def __enter__(self):
+        if self.ok:
+            self.t = threading.Thread(target=self._run, daemon=True)
+            self.t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        if self.ok:
+            self.t.join()
+
+    def summary(self):
+        if not self.ok:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvml unavailable"]}
+        return {"sm_mhz": float(np.median(self.samples)) if self.samples else None, "sm_max_mhz": self.max_mhz,
+                "samples": len(self.samples),
+                "reasons": [n for b, n in self.REASONS.items() if self.reasons & b]}
+
+
+# --------------------------------------------------------------------------
+# CPU oracle (cpu_baseline leg and --impl reference)
+# --------------------------------------------------------------------------
+def sample_rows(A_h, n_rows, seed=0):
+    rng = np.random.default_rng(seed)
+    rows = np.sort(rng.choice(A_h.n_rows, size=min(n_rows, A_h.n_rows), replace=False))
+    l = np.diff(A_h.row_ptr)[rows]
+    rp = np.concatenate([[0], np.cumsum(l)]).astype(np.int64)
+    idx = np.concatenate([np.arange(A_h.row_ptr[r], A_h.row_ptr[r + 1]) for r in rows]) if len(rows) else \
+        np.zeros(0, np.int64)
+    return gen.CSR(len(rows), A_h.n_cols, rp, A_h.col_ind[idx], A_h.val[idx], A_h.name + "-sample")
+
+
+def oracle_step(sub, B_h, J):
+    """The oracle of the whole path on a row sample: Algorithm 3 over eq. 7
+    (configure), CSR->CELL, Algorithm 2 SpMM -- all single-threaded C."""
+    import oracle
+    e, k = oracle.configure(sub, 1, J)
+    cell = oracle.csr_to_cell(sub, 1, e, k)
+    oracle.cell_spmm(cell, B_h)
+
+
+def calibrate_sample(A_h, B_h, J, target_s):
+    n = max(64, A_h.n_rows // 2000)
+    while True:
+        sub = sample_rows(A_h, n)
+        t0 = time.perf_counter()
+        oracle_step(sub, B_h, J)
+        dt = time.perf_counter() - t0
+        if dt > 0.3 or n >= A_h.n_rows:
+            break
+        n = min(A_h.n_rows, n * 4)
+    n = int(min(A_h.n_rows, max(64, n * target_s / max(dt, 1e-6))))
+    return sample_rows(A_h, n)
+
+
+def cpu_baseline(A_h, B_h, J, target_s=15.0):
+    sub = calibrate_sample(A_h, B_h, J, target_s)
+    t0 = time.perf_counter()
+    oracle_step(sub, B_h, J)
+    dt = time.perf_counter() - t0
+    return {"value": 2.0 * sub.nnz * J / dt / 1e9, "unit": "GFLOP/s", "cores": 1, "kind": "oracle",
+            "sample": f"{sub.n_rows} random rows ({sub.nnz} nnz) of the workload; oracle configure (Alg. 3 over "
+                      f"eq. 7) + CSR->CELL + Alg. 2 fp64 SpMM, single thread, {dt:.2f} s",
+            "host_cpus": os.cpu_count()}
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return 0
+    A_h, J = gen.config(args.config, args.seed)
+    B_h = gen.dense(A_h.n_cols, J, args.seed)
+    per_step = max(0.2, min(5.0, 120.0 / (args.steps + args.warmup)))
+    sub = calibrate_sample(A_h, B_h, J, per_step)
+    for _ in range(args.warmup):
+        oracle_step(sub, B_h, J)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        oracle_step(sub, B_h, J)
+    dt = (time.perf_counter() - t0) / args.steps
+    v = 2.0 * sub.nnz * J / dt / 1e9
+    line = {"metric": METRIC, "value": v, "unit": "GFLOP/s", "impl": "reference", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
+            "config": {"workload": args.config, "J": J, "n_rows": A_h.n_rows, "nnz": A_h.nnz,
+                       "sample_rows": sub.n_rows, "sample_nnz": sub.nnz},
+            "cpu_baseline": {"value": v, "unit": "GFLOP/s", "cores": 1, "kind": "oracle",
+                             "sample": f"{sub.n_rows} random rows ({sub.nnz} nnz) per step; oracle configure + "
+                                       "CSR->CELL + Alg. 2 fp64, single thread"},
+            "e2e": {"value": v, "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# --------------------------------------------------------------------------
+# GPU arm
+# --------------------------------------------------------------------------
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--config", default="c2_rmat20")
+    ap.add_argument("--seed", type=int, default=0)
+    ap.add_argument("--parts", type=int, default=0, help="force P (0 = predictor stand-in)")
+    ap.add_argument("--width-log2", type=int, default=-1, help="force e_p (-1 = Algorithm 3)")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--shard-mode", default="nnz", choices=["nnz", "bytes"])
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import torch
+    import torch.distributed as dist
+    import paper_conf_hpdc_pengtpk25_b200 as lf
+    from paper_conf_hpdc_pengtpk25_b200 import dist as lfd
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+
+    A_h, J = gen.config(args.config, args.seed)
+    B_h = gen.dense(A_h.n_cols, J, args.seed)
+    bytes_alg, U = algorithmic_bytes(A_h, J)
+    flops = 2.0 * A_h.nnz * J
+    bounds = lfd.shard_bounds(A_h.row_ptr, world, J, args.shard_mode)
+    lo, hi = int(bounds[rank]), int(bounds[rank + 1])
+    p0, p1 = int(A_h.row_ptr[lo]), int(A_h.row_ptr[hi])
+    # host (pinned) copies of this rank's shard -- the e2e leg copies them every step
+    h_rp = torch.from_numpy(A_h.row_ptr[lo:hi + 1] - p0).pin_memory()
+    h_ci = torch.from_numpy(A_h.col_ind[p0:p1]).pin_memory()
+    h_va = torch.from_numpy(A_h.val[p0:p1]).pin_memory()
+    h_B = torch.from_numpy(B_h).pin_memory()
+    d_rp, d_ci, d_va, d_B = (t.to(dev) for t in (h_rp, h_ci, h_va, h_B))
+    A = lf.Csr(d_rp, d_ci, d_va, A_h.n_cols, p1 - p0)
+    I_loc = hi - lo
+    C_loc = torch.empty((I_loc, J), dtype=torch.float32, device=dev)
+    h_C = torch.empty((I_loc, J), dtype=torch.float32).pin_memory()
+    stream = torch.cuda.current_stream()
+    kw = {}
+    if args.parts:
+        kw["force_parts"] = args.parts
+    if args.width_log2 >= 0:
+        kw["force_width_log2"] = args.width_log2
+
+    ev = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
+    phase = {"configure": [], "build": [], "spmm": [], "gather": []}
+    info = {}
+
+    def step(Ain, record=False):
+        e0 = ev(); e0.record(stream)
+        params, stats = lf.configure(Ain, J, **kw)
+        e1 = ev(); e1.record(stream)
+        M = lf.CellMatrix.build(Ain, params)
+        e2 = ev(); e2.record(stream)
+        M.spmm(d_B, out=C_loc)
+        e3 = ev(); e3.record(stream)
+        if world > 1:
+            lfd.gather_rows(C_loc, bounds)
+        e4 = ev(); e4.record(stream)
+        if record:
+            phase["_ev"].append((e0, e1, e2, e3, e4))
+            info["params"] = params.as_dict()
+            v = M.view()
+            info["cell_slots"] = int(v["n_slots"])
+            info["cell_rows"] = int(v["n_cell_rows"])
+            info["n_buckets"] = len(v["buckets"])
+        M.close()
+        return params
+
+    phase["_ev"] = []
+    for _ in range(args.warmup):
+        step(A)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    with ClockSampler(local) as clk:
+        t0 = ev(); t1 = ev()
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+        t0.record(stream)
+        for _ in range(args.steps):
+            params = step(A, record=True)
+        t1.record(stream)
+        torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    ms = t0.elapsed_time(t1) / args.steps
+    for (e0, e1, e2, e3, e4) in phase["_ev"]:
+        phase["configure"].append(e0.elapsed_time(e1))
+        phase["build"].append(e1.elapsed_time(e2))
+        phase["spmm"].append(e2.elapsed_time(e3))
+        phase["gather"].append(e3.elapsed_time(e4))
+    ph = {k: float(np.mean(v)) for k, v in phase.items() if k != "_ev"}
+
+    def maxr(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    ms = maxr(ms)
+    ph = {k: maxr(v) for k, v in ph.items()}
+
+    # ---- SpMM alone (the paper's kernel-only time) -----------
+    params, _ = lf.configure(A, J, **kw)
+    M = lf.CellMatrix.build(A, params)
+    for _ in range(3):
+        M.spmm(d_B, out=C_loc)
+    torch.cuda.synchronize()
+    n_sp = max(10, args.steps)
+    s0, s1 = ev(), ev()
+    s0.record(stream)
+    for _ in range(n_sp):
+        M.spmm(d_B, out=C_loc)
+    s1.record(stream)
+    torch.cuda.synchronize()
+    spmm_ms = maxr(s0.elapsed_time(s1) / n_sp)
+
+    # ---- e2e: host buffers in, result back, through the public API ---------
+    e2e = None
+    if not args.no_e2e:
+        h2d = sum(t.numel() * t.element_size() for t in (h_rp, h_ci, h_va, h_B))
+        d2h = h_C.numel() * 4
+
+        def e2e_step():
+            for hs, ds in ((h_rp, d_rp), (h_ci, d_ci), (h_va, d_va), (h_B, d_B)):
+                ds.copy_(hs, non_blocking=True)
+            Ain = lf.Csr(d_rp, d_ci, d_va, A_h.n_cols, p1 - p0)
+            pr, _ = lf.configure(Ain, J, **kw)
+            Mi = lf.CellMatrix.build(Ain, pr)
+            Mi.spmm(d_B, out=C_loc)
+            if world > 1:
+                lfd.gather_rows(C_loc, bounds)
+            h_C.copy_(C_loc, non_blocking=True)
+            Mi.close()
+
+        for _ in range(2):
+            e2e_step()
+        torch.cuda.synchronize()
+        x0, x1 = ev(), ev()
+        x0.record(stream)
+        n_e2e = max(3, min(args.steps, 20))
+        for _ in range(n_e2e):
+            e2e_step()
+        x1.record(stream)
+        torch.cuda.synchronize()
+        e2e_ms = maxr(x0.elapsed_time(x1) / n_e2e)
+        e2e = {"value": flops / (e2e_ms * 1e-3) / 1e9, "unit": "GFLOP/s", "ms_per_step": e2e_ms,
+               "h2d_bytes_per_step": int(h2d * world), "d2h_bytes_per_step": int(d2h * world)}
+
+    if rank != 0:
+        if world > 1:
+            dist.destroy_process_group()
+        return 0
+    hbm_peak, peak_kind = peaks()
+    P = params.n_parts
+    launches_per_step = 2 + (4 + (1 if P > 1 else 0)) + 2
+    sp_ms = ph["spmm"]
+    line = {
+        "metric": METRIC, "value": flops / (ms * 1e-3) / 1e9, "unit": "GFLOP/s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+        "config": {"workload": args.config, "J": J, "n_rows": A_h.n_rows, "n_cols": A_h.n_cols, "nnz": A_h.nnz,
+                   "distinct_cols": U, "params": info.get("params"), "cell_slots": info.get("cell_slots"),
+                   "cell_rows": info.get("cell_rows"), "n_buckets": info.get("n_buckets"),
+                   "parallelism": f"rows{world}", "shard_mode": args.shard_mode,
+                   "l2": "inputs larger than L2 (B, C, CELL each >126 MB); no flush"},
+        "phases_ms": ph,
+        "spmm_only": {"ms": spmm_ms, "gflops": flops / (spmm_ms * 1e-3) / 1e9,
+                      "hbm_gbs_alg": bytes_alg / (spmm_ms * 1e-3) / 1e9},
+        "roofline": {"kernel": "lf_spmm (zero_rows + cell_spmm_kernel)", "bound": "hbm",
+                     "achieved": bytes_alg / world / (sp_ms * 1e-3) / 1e9, "peak": hbm_peak, "unit": "GB/s",
+                     "frac": bytes_alg / world / (sp_ms * 1e-3) / 1e9 / hbm_peak, "peak_kind": peak_kind,
+                     "bytes_alg_per_launch": bytes_alg // world, "traffic": None},
+        "clocks": clk.summary(),
+        "gpu_launches": launches_per_step * args.steps,
+        "e2e": e2e,
+    }
+    if world == 1 and not args.no_cpu_baseline:
+        line["cpu_baseline"] = cpu_baseline(A_h, B_h, J)
+    print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.destroy_process_group()
+    return 0
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,424 @@
+// lf_api.cu -- the C ABI of liblf.so (include/liteform.h): argument checks,
+// handle and memory management, the host side of configure (eq. 7 +
+// Algorithm 3 over GPU statistics) and of the CSR -> CELL build.
+#include <algorithm>
+#include <cmath>
+#include <cstdlib>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "lf_internal.cuh"
+
+namespace {
+
+thread_local std::string g_detail;
+
+lf_status fail(lf_status st, const std::string &why) {
+    g_detail = why;
+    return st;
+}
+
+#define LF_CUDA(expr)                                                                          \
+    do {                                                                                       \
+        cudaError_t e_ = (expr);                                                               \
+        if (e_ != cudaSuccess) return fail(LF_ERR_CUDA, std::string(#expr) + ": " + cudaGetErrorString(e_)); \
+    } while (0)
+
+// ---- memory -------------------------------------------------------------
+struct Mem {
+    const lf_allocator *al;
+    cudaStream_t s;
+    void *get(size_t bytes) {
+        if (bytes == 0) return nullptr;
+        bytes = (bytes + 255) & ~size_t(255);
+        if (al && al->alloc) return al->alloc(al->ctx, bytes, s);
+        void *p = nullptr;
+        if (cudaMallocAsync(&p, bytes, s) != cudaSuccess) return nullptr;
+        return p;
+    }
+    void put(void *p, size_t bytes) {
+        if (!p) return;
+        bytes = (bytes + 255) & ~size_t(255);
+        if (al && al->free) al->free(al->ctx, p, bytes, s);
+        else cudaFreeAsync(p, s);
+    }
+};
+
+// RAII list of allocations released at scope exit (scratch)
+struct Scratch {
+    Mem m;
+    std::vector<std::pair<void *, size_t>> v;
+    template <typename T>
+    T *get(size_t n) {
+        void *p = m.get(n * sizeof(T));
+        if (n && p) v.push_back({p, n * sizeof(T)});
+        return static_cast<T *>(p);
+    }
+    ~Scratch() {
+        for (auto &x : v) m.put(x.first, x.second);
+    }
+};
+
+lf_status check_csr(const lf_csr *A) {
+    if (!A) return fail(LF_ERR_INVALID_ARG, "A is NULL");
+    if (A->n_rows < 0 || A->n_cols < 0 || A->nnz < 0) return fail(LF_ERR_INVALID_ARG, "negative size");
+    if (!A->row_ptr) return fail(LF_ERR_INVALID_ARG, "row_ptr is NULL");
+    if (A->nnz > 0 && (!A->col_ind || !A->val)) return fail(LF_ERR_INVALID_ARG, "col_ind/val NULL with nnz > 0");
+    if (A->n_cols > 2147483647LL) return fail(LF_ERR_INDEX_OVERFLOW, "n_cols exceeds int32");
+    if (A->n_rows >= (int64_t(1) << 30)) return fail(LF_ERR_INDEX_OVERFLOW, "n_rows >= 2^30");
+    return LF_OK;
+}
+
+lf_status maybe_validate(const lf_csr *A, cudaStream_t s) {
+    const char *v = std::getenv("LF_VALIDATE");
+    if (!v || v[0] != '1' || A->n_rows == 0) return LF_OK;
+    int *d_flag = nullptr;
+    LF_CUDA(cudaMallocAsync(&d_flag, sizeof(int), s));
+    LF_CUDA(cudaMemsetAsync(d_flag, 0, sizeof(int), s));
+    LF_CUDA(lf::launch_validate(*A, d_flag, s));
+    int flag = 0;
+    LF_CUDA(cudaMemcpyAsync(&flag, d_flag, sizeof(int), cudaMemcpyDeviceToHost, s));
+    LF_CUDA(cudaFreeAsync(d_flag, s));
+    LF_CUDA(cudaStreamSynchronize(s));
+    if (flag & 2) return fail(LF_ERR_INVALID_ARG, "column index out of range or row_ptr decreasing");
+    if (flag & 1) return fail(LF_ERR_UNSORTED_CSR, "columns not sorted within a row");
+    return LF_OK;
+}
+
+// Predictor slot (sections 5.1-5.2).  No trained model exists
+// for this hardware (parity unpinned): the stand-in
+// chooses CELL and P = 1.
+int standin_parts(const lf_csr *A, int32_t J, int max_parts) {
+    (void)A;
+    (void)J;
+    return std::max(1, std::min(1, max_parts));
+}
+
+// Algorithm 3 in exponent space (reading R8) over eq. 7 costs.
+int alg3(const int64_t *cost, int hi) {
+    int lo = 0;
+    while (lo < hi) {
+        int mid = (lo + hi) / 2;
+        if (cost[mid] > cost[mid + 1]) lo = mid + 1;
+        else hi = mid;
+    }
+    return lo;
+}
+
+}  // namespace
+
+extern "C" {
+
+int32_t lf_abi_version(void) { return LF_ABI_VERSION; }
+
+const char *lf_status_string(lf_status st) {
+    switch (st) {
+    case LF_OK: return "LF_OK";
+    case LF_ERR_INVALID_ARG: return "LF_ERR_INVALID_ARG";
+    case LF_ERR_UNSORTED_CSR: return "LF_ERR_UNSORTED_CSR";
+    case LF_ERR_INDEX_OVERFLOW: return "LF_ERR_INDEX_OVERFLOW";
+    case LF_ERR_NO_MEMORY: return "LF_ERR_NO_MEMORY";
+    case LF_ERR_CUDA: return "LF_ERR_CUDA";
+    case LF_ERR_UNSUPPORTED: return "LF_ERR_UNSUPPORTED";
+    }
+    return "LF_ERR_UNKNOWN";
+}
+
+const char *lf_last_error_detail(void) { return g_detail.c_str(); }
+
+lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts *opts, lf_cell_params *out,
+                            lf_configure_stats *stats, lf_stream_t stream) {
+    g_detail.clear();
+    if (lf_status st = check_csr(A)) return st;
+    if (!out) return fail(LF_ERR_INVALID_ARG, "out is NULL");
+    if (J < 1) return fail(LF_ERR_INVALID_ARG, "J < 1");
+    lf_configure_opts o{};
+    if (opts) o = *opts;
+    if (o.max_parts < 0 || o.max_parts > LF_MAX_PARTS) return fail(LF_ERR_INVALID_ARG, "max_parts out of range");
+    if (o.block_mult_log2 < 0 || o.block_mult_log2 > LF_MAX_LOG2) return fail(LF_ERR_INVALID_ARG, "block_mult_log2");
+    if (o.force_parts < 0 || o.force_parts > LF_MAX_PARTS) return fail(LF_ERR_INVALID_ARG, "force_parts");
+    if (o.force_width_log2 > LF_MAX_LOG2) return fail(LF_ERR_INVALID_ARG, "force_width_log2");
+    if (o.force_format < 0 || o.force_format > 2) return fail(LF_ERR_INVALID_ARG, "force_format");
+    const int max_parts = o.max_parts ? o.max_parts : LF_MAX_PARTS;
+    cudaStream_t s = (cudaStream_t)stream;
+    if (lf_status st = maybe_validate(A, s)) return st;
+
+    const int P = o.force_parts ? o.force_parts : standin_parts(A, J, max_parts);
+    lf::StatsDev *d_st = nullptr;
+    uint32_t *d_mask = nullptr;
+    LF_CUDA(cudaMallocAsync(&d_st, sizeof(lf::StatsDev), s));
+    LF_CUDA(cudaMemsetAsync(d_st, 0, sizeof(lf::StatsDev), s));
+    LF_CUDA(cudaMemsetAsync(&d_st->len_min, 0xFF, sizeof(unsigned long long), s));
+    if (A->n_cols > 0) {
+        LF_CUDA(cudaMallocAsync(&d_mask, (size_t)A->n_cols * sizeof(uint32_t), s));
+        LF_CUDA(cudaMemsetAsync(d_mask, 0, (size_t)A->n_cols * sizeof(uint32_t), s));
+    }
+    LF_CUDA(lf::launch_stats(*A, P, d_st, d_mask, s));
+    std::vector<lf::StatsDev> h(1);
+    LF_CUDA(cudaMemcpyAsync(h.data(), d_st, sizeof(lf::StatsDev), cudaMemcpyDeviceToHost, s));
+    LF_CUDA(cudaFreeAsync(d_st, s));
+    if (d_mask) LF_CUDA(cudaFreeAsync(d_mask, s));
+    LF_CUDA(cudaStreamSynchronize(s));
+    const lf::StatsDev &st = h[0];
+
+    lf_configure_stats local;
+    lf_configure_stats &cs = stats ? *stats : local;
+    std::memset(&cs, 0, sizeof(cs));
+    const double I = (double)A->n_rows;
+    const double mean = A->n_rows ? (double)st.len_sum / I : 0.0;
+    double var = A->n_rows ? (double)st.len_sumsq / I - mean * mean : 0.0;
+    cs.features[0] = I;
+    cs.features[1] = (double)A->n_cols;
+    cs.features[2] = (double)st.len_sum;
+    cs.features[3] = mean;
+    cs.features[4] = A->n_rows ? (double)st.len_min : 0.0;
+    cs.features[5] = (double)st.len_max;
+    cs.features[6] = var > 0 ? std::sqrt(var) : 0.0;
+    cs.features[7] = (double)J;
+    cs.n_parts = P;
+
+    lf_cell_params prm{};
+    prm.use_cell = o.force_format == 2 ? 0 : 1;
+    prm.n_parts = P;
+    for (int p = 0; p < P; p++) {
+        int top = -1;
+        for (int t = 0; t < lf::kMaxT; t++) {
+            cs.H[p][t] = (int64_t)st.H[p][t];
+            cs.F[p][t] = (int64_t)st.F[p][t];
+            cs.Unat[p][t] = (int64_t)st.Unat[p][t];
+            cs.Utop[p][t] = (int64_t)st.Utop[p][t];
+            cs.cost[p][t] = -1;
+            if (st.H[p][t]) top = t;
+        }
+        cs.max_log2[p] = top;
+        // eq. 7 (reading R10): buckets b < e keep their natural rows,
+        // the max bucket e holds every row with ceil_log2 l >= e, folded.
+        for (int e = 0; e <= top; e++) {
+            int64_t c = 0;
+            for (int b = 0; b < e; b++)
+                if (cs.H[p][b]) c += 2 * cs.H[p][b] * (int64_t(1) << b) + cs.Unat[p][b] * J + cs.H[p][b] * J;
+            if (cs.F[p][e]) c += 2 * cs.F[p][e] * (int64_t(1) << e) + cs.Utop[p][e] * J + cs.F[p][e] * J;
+            cs.cost[p][e] = c;
+        }
+        int e;
+        if (top < 0) e = 0;
+        else if (o.force_width_log2 >= 0) e = std::min(o.force_width_log2, top);
+        else e = alg3(cs.cost[p], top);
+        cs.chosen_log2[p] = top < 0 ? -1 : e;
+        prm.max_width_log2[p] = (int8_t)e;
+        prm.block_nnz_log2[p] = (int8_t)std::min(e + o.block_mult_log2, LF_MAX_LOG2);
+    }
+    *out = prm;
+    return LF_OK;
+}
+
+lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_allocator *al, lf_stream_t stream,
+                        lf_cell **out) {
+    g_detail.clear();
+    if (lf_status st = check_csr(A)) return st;
+    if (!params || !out) return fail(LF_ERR_INVALID_ARG, "params/out is NULL");
+    *out = nullptr;
+    const int P = params->n_parts;
+    if (P < 1 || P > LF_MAX_PARTS) return fail(LF_ERR_INVALID_ARG, "n_parts out of range");
+    if (params->use_cell != 0 && params->use_cell != 1) return fail(LF_ERR_INVALID_ARG, "use_cell");
+    for (int p = 0; p < P; p++) {
+        const int e = params->max_width_log2[p], k = params->block_nnz_log2[p];
+        if (e < 0 || e > LF_MAX_LOG2 || k < e || k > LF_MAX_LOG2)
+            return fail(LF_ERR_INVALID_ARG, "need 0 <= e_p <= k_p <= 30");
+    }
+    if (al && (!al->alloc || !al->free)) return fail(LF_ERR_INVALID_ARG, "allocator without alloc/free");
+    cudaStream_t s = (cudaStream_t)stream;
+    if (lf_status st = maybe_validate(A, s)) return st;
+
+    lf_cell *h = new lf_cell();
+    h->params = *params;
+    h->n_rows = A->n_rows;
+    h->n_cols = A->n_cols;
+    h->nnz = A->nnz;
+    h->stream = s;
+    if (al) {
+        h->al = *al;
+        h->custom_al = true;
+    }
+    auto bail = [&](lf_status st) {
+        lf_cell_destroy(h);
+        return st;
+    };
+    if (params->use_cell == 0) {  // fixed format: keep the caller's CSR
+        h->csr = *A;
+        *out = h;
+        return LF_OK;
+    }
+    Mem mem{al, s};
+    const int64_t I = A->n_rows;
+    const int n_tiles = (int)((I + lf::kBuildTile - 1) / lf::kBuildTile);
+    Scratch sc{mem, {}};
+    lf::BuildScratch bs{};
+    bs.n_tiles = n_tiles;
+    int8_t *d_e = sc.get<int8_t>(LF_MAX_PARTS);
+    bs.seg_rel = P > 1 ? sc.get<int32_t>((size_t)I * (P - 1)) : nullptr;
+    bs.tile_cnt = sc.get<long long>((size_t)P * lf::kMaxT * std::max(n_tiles, 1));
+    bs.key_total = sc.get<long long>((size_t)P * lf::kMaxT);
+    bs.key_row_off = sc.get<long long>((size_t)P * lf::kMaxT);
+    h->row_cnt = static_cast<int32_t *>(mem.get((size_t)std::max<int64_t>(I, 1) * sizeof(int32_t)));
+    if (!d_e || !bs.tile_cnt || !bs.key_total || !bs.key_row_off || !h->row_cnt || (P > 1 && I > 0 && !bs.seg_rel))
+        return bail(fail(LF_ERR_NO_MEMORY, "scratch allocation failed"));
+
+    // a1 + a4 (count): segments, bucket keys, per-tile totals, tile scan
+    auto cu = [&](cudaError_t e, const char *what) -> lf_status {
+        if (e != cudaSuccess) return fail(LF_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
+        return LF_OK;
+    };
+    lf_status st;
+    if ((st = cu(cudaMemcpyAsync(d_e, params->max_width_log2, LF_MAX_PARTS, cudaMemcpyHostToDevice, s), "H2D e")))
+        return bail(st);
+    if ((st = cu(cudaMemsetAsync(h->row_cnt, 0, (size_t)std::max<int64_t>(I, 1) * sizeof(int32_t), s), "memset")))
+        return bail(st);
+    if ((st = cu(cudaMemsetAsync(bs.tile_cnt, 0, (size_t)P * lf::kMaxT * std::max(n_tiles, 1) * 8, s), "memset")))
+        return bail(st);
+    if ((st = cu(lf::launch_seg(*A, P, bs.seg_rel, s), "seg"))) return bail(st);
+    if ((st = cu(lf::launch_bucket_count(*A, P, d_e, bs, h->row_cnt, s), "bucket_count"))) return bail(st);
+    if (n_tiles > 0 && (st = cu(lf::launch_tile_scan(P, bs, s), "tile_scan"))) return bail(st);
+    std::vector<long long> tot((size_t)P * lf::kMaxT, 0);
+    if (n_tiles > 0 &&
+        (st = cu(cudaMemcpyAsync(tot.data(), bs.key_total, tot.size() * 8, cudaMemcpyDeviceToHost, s), "D2H")))
+        return bail(st);
+    if ((st = cu(cudaStreamSynchronize(s), "sync"))) return bail(st);
+
+    // host: bucket table (R2, R7) and warp-task decomposition
+    std::vector<long long> row_off((size_t)P * lf::kMaxT, -1);
+    int64_t R_tot = 0, S_tot = 0, tasks = 0;
+    for (int p = 0; p < P; p++) {
+        const int k = params->block_nnz_log2[p];
+        for (int t = 0; t <= params->max_width_log2[p]; t++) {
+            const long long n = tot[(size_t)p * lf::kMaxT + t];
+            if (n == 0) continue;
+            const int64_t R = int64_t(1) << (k - t), W = int64_t(1) << t;
+            const int64_t pad = (n + R - 1) / R * R;
+            lf_bucket b{};
+            b.part = p;
+            b.width_log2 = t;
+            b.rows_per_block = (int32_t)std::min<int64_t>(R, INT32_MAX);
+            b.n_rows = n;
+            b.n_rows_pad = pad;
+            b.row_off = R_tot;
+            b.slot_off = S_tot;
+            h->buckets.push_back(b);
+            lf::BucketDev d{};
+            d.slot_off = S_tot;
+            d.row_off = R_tot;
+            d.n_slots = pad * W;
+            d.task_off = tasks;
+            d.t = t;
+            d.task_slots = (int32_t)std::max<int64_t>(32, W);
+            h->h_buckets.push_back(d);
+            row_off[(size_t)p * lf::kMaxT + t] = R_tot;
+            tasks += W <= 32 ? (pad * W + 31) / 32 : pad;
+            R_tot += pad;
+            S_tot += pad * W;
+        }
+    }
+    h->n_cell_rows = R_tot;
+    h->n_slots = S_tot;
+    h->n_tasks = tasks;
+    const int nb = (int)h->buckets.size();
+    if (nb > 2048) return bail(fail(LF_ERR_UNSUPPORTED, "more than 2048 buckets"));
+
+    // persistent arrays: one pool
+    const size_t a256 = 256;
+    auto up = [&](size_t b) { return (b + a256 - 1) / a256 * a256; };
+    const size_t b_ri = up(R_tot * 4), b_rt = up(R_tot * 4), b_ci = up(S_tot * 4), b_va = up(S_tot * 4),
+                 b_bk = up(nb * sizeof(lf::BucketDev));
+    h->pool_bytes = b_ri + b_rt + b_ci + b_va + b_bk;
+    h->pool = mem.get(h->pool_bytes);
+    if (h->pool_bytes && !h->pool) return bail(fail(LF_ERR_NO_MEMORY, "CELL arrays allocation failed"));
+    char *q = static_cast<char *>(h->pool);
+    h->row_ind = reinterpret_cast<int32_t *>(q);
+    h->row_tag = reinterpret_cast<int32_t *>(q + b_ri);
+    h->col_ind = reinterpret_cast<int32_t *>(q + b_ri + b_rt);
+    h->val = reinterpret_cast<float *>(q + b_ri + b_rt + b_ci);
+    h->d_buckets = reinterpret_cast<lf::BucketDev *>(q + b_ri + b_rt + b_ci + b_va);
+    bs.src_pos = sc.get<int64_t>((size_t)R_tot);
+    bs.src_cnt = sc.get<int32_t>((size_t)R_tot);
+    if (R_tot && (!bs.src_pos || !bs.src_cnt)) return bail(fail(LF_ERR_NO_MEMORY, "scratch allocation failed"));
+
+    if (R_tot) {
+        if ((st = cu(cudaMemsetAsync(h->row_ind, 0xFF, R_tot * 4, s), "memset"))) return bail(st);
+        if ((st = cu(cudaMemsetAsync(h->row_tag, 0xFF, R_tot * 4, s), "memset"))) return bail(st);
+        if ((st = cu(cudaMemsetAsync(bs.src_cnt, 0, R_tot * 4, s), "memset"))) return bail(st);
+    }
+    if (nb && (st = cu(cudaMemcpyAsync(h->d_buckets, h->h_buckets.data(), nb * sizeof(lf::BucketDev),
+                                       cudaMemcpyHostToDevice, s),
+                       "H2D buckets")))
+        return bail(st);
+    if ((st = cu(cudaMemcpyAsync(bs.key_row_off, row_off.data(), row_off.size() * 8, cudaMemcpyHostToDevice, s),
+                 "H2D row_off")))
+        return bail(st);
+    // a4 (place) + a5 (scatter)
+    if ((st = cu(lf::launch_bucket_place(*A, P, d_e, bs, h->row_cnt, h->row_ind, h->row_tag, s), "bucket_place")))
+        return bail(st);
+    if ((st = cu(lf::launch_slot_fill(*A, h->d_buckets, nb, S_tot, bs, h->col_ind, h->val, s), "slot_fill")))
+        return bail(st);
+    *out = h;
+    return LF_OK;
+}
+
+lf_status lf_spmm(const lf_cell *h, const float *B, int64_t ldb, int32_t J, float *C, int64_t ldc,
+                  lf_stream_t stream) {
+    g_detail.clear();
+    if (!h) return fail(LF_ERR_INVALID_ARG, "handle is NULL");
+    if (J < 0 || ldb < J || ldc < J || ldb < 0 || ldc < 0) return fail(LF_ERR_INVALID_ARG, "need 0 <= J <= ldb, ldc");
+    if (J == 0 || h->n_rows == 0) return LF_OK;
+    if (!C) return fail(LF_ERR_INVALID_ARG, "C is NULL");
+    if (!B && h->n_cols > 0) return fail(LF_ERR_INVALID_ARG, "B is NULL");
+    cudaStream_t s = (cudaStream_t)stream;
+    if (h->params.use_cell == 0) {
+        LF_CUDA(lf::launch_csr_spmm(h->csr, B, ldb, J, C, ldc, s));
+        return LF_OK;
+    }
+    LF_CUDA(lf::launch_zero_rows(h->row_cnt, h->n_rows, C, ldc, J, s));
+    lf::SpmmArgs a{h->d_buckets, (int)h->buckets.size(), h->n_tasks, h->col_ind, h->val, h->row_tag,
+                   B, ldb, C, ldc, J};
+    LF_CUDA(lf::launch_cell_spmm(a, s));
+    return LF_OK;
+}
+
+lf_status lf_csr_spmm(const lf_csr *A, const float *B, int64_t ldb, int32_t J, float *C, int64_t ldc,
+                      lf_stream_t stream) {
+    g_detail.clear();
+    if (lf_status st = check_csr(A)) return st;
+    if (J < 0 || ldb < J || ldc < J) return fail(LF_ERR_INVALID_ARG, "need 0 <= J <= ldb, ldc");
+    if (J == 0 || A->n_rows == 0) return LF_OK;
+    if (!C || (!B && A->n_cols > 0)) return fail(LF_ERR_INVALID_ARG, "B/C is NULL");
+    LF_CUDA(lf::launch_csr_spmm(*A, B, ldb, J, C, ldc, (cudaStream_t)stream));
+    return LF_OK;
+}
+
+lf_status lf_cell_view(const lf_cell *h, lf_cell_arrays *out) {
+    if (!h || !out) return fail(LF_ERR_INVALID_ARG, "NULL argument");
+    std::memset(out, 0, sizeof(*out));
+    out->n_rows = h->n_rows;
+    out->n_cols = h->n_cols;
+    out->nnz = h->nnz;
+    out->n_cell_rows = h->n_cell_rows;
+    out->n_slots = h->n_slots;
+    out->n_buckets = (int32_t)h->buckets.size();
+    out->row_ind = h->row_ind;
+    out->col_ind = h->col_ind;
+    out->val = h->val;
+    out->buckets = h->buckets.empty() ? nullptr : h->buckets.data();
+    out->params = h->params;
+    return LF_OK;
+}
+
+lf_status lf_cell_destroy(lf_cell *h) {
+    if (!h) return LF_OK;
+    Mem mem{h->custom_al ? &h->al : nullptr, h->stream};
+    mem.put(h->pool, h->pool_bytes);
+    mem.put(h->row_cnt, (size_t)std::max<int64_t>(h->n_rows, 1) * sizeof(int32_t));
+    delete h;
+    return LF_OK;
+}
+
+}  // extern "C"

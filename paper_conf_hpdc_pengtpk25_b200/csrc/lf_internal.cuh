@@ -1,0 +1,112 @@
+// lf_internal.cuh -- internal declarations shared by liblf.so's translation
+// units (never included by the oracle; never exported).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "liteform.h"
+
+namespace lf {
+
+constexpr int kMaxT = 32;  // natural buckets t = 0..31
+
+// ceil(log2(l)) for l >= 1 (natural bucket, reading R1)
+__host__ __device__ __forceinline__ int ceil_log2_i64(int64_t l) {
+#ifdef __CUDA_ARCH__
+    return l <= 1 ? 0 : 64 - __clzll((unsigned long long)(l - 1));
+#else
+    int t = 0;
+    while ((int64_t(1) << t) < l) t++;
+    return t;
+#endif
+}
+
+// Per-bucket descriptor the SpMM kernel walks (device copy of the bucket
+// table plus its work decomposition into warp tasks).
+struct BucketDev {
+    int64_t slot_off;   // first slot
+    int64_t row_off;    // first CELL row
+    int64_t n_slots;    // n_rows_pad * W
+    int64_t task_off;   // first task index of this bucket
+    int32_t t;          // log2 width
+    int32_t task_slots; // slots per task: 32 (W <= 32) or W (one row per task)
+};
+
+// Stats the configure kernels accumulate (device, zero-initialised).
+struct StatsDev {
+    unsigned long long len_min, len_max, len_sum, len_sumsq;  // row lengths
+    unsigned long long H[LF_MAX_PARTS][kMaxT];
+    unsigned long long F[LF_MAX_PARTS][kMaxT];
+    unsigned long long Unat[LF_MAX_PARTS][kMaxT];
+    unsigned long long Utop[LF_MAX_PARTS][kMaxT];
+};
+
+// ---- launchers (kernels in csrc/kernels/*.cu) ----
+cudaError_t launch_stats(const lf_csr &A, int P, StatsDev *d_stats, uint32_t *d_colmask, cudaStream_t s);
+
+struct BuildScratch {
+    int32_t *seg_rel;       // [I*(P-1)] segment starts relative to the row start (P > 1)
+    long long *tile_cnt;    // [P][n_tiles][32] n_sub sums per tile -> exclusive offsets
+    long long *key_total;   // [P][32]
+    long long *key_row_off; // [P][32] first CELL row of bucket (p,t), -1 if none
+    int64_t *src_pos;       // [R_tot] CSR position of a CELL row's first slot
+    int32_t *src_cnt;       // [R_tot] real slots in the CELL row (0 for padding)
+    int n_tiles;
+};
+constexpr int kBuildTile = 256;  // rows per tile of the bucketize passes
+
+cudaError_t launch_seg(const lf_csr &A, int P, int32_t *seg_rel, cudaStream_t s);
+cudaError_t launch_bucket_count(const lf_csr &A, int P, const int8_t *e, const BuildScratch &sc,
+                                int32_t *row_cnt, cudaStream_t s);
+cudaError_t launch_tile_scan(int P, const BuildScratch &sc, cudaStream_t s);
+cudaError_t launch_bucket_place(const lf_csr &A, int P, const int8_t *e, const BuildScratch &sc,
+                                const int32_t *row_cnt, int32_t *row_ind, int32_t *row_tag, cudaStream_t s);
+cudaError_t launch_slot_fill(const lf_csr &A, const BucketDev *d_buckets, int nb, int64_t n_slots,
+                             const BuildScratch &sc, int32_t *col_out, float *val_out, cudaStream_t s);
+
+// SpMM
+struct SpmmArgs {
+    const BucketDev *buckets;
+    int nb;
+    int64_t n_tasks;
+    const int32_t *col;
+    const float *val;
+    const int32_t *row_tag;
+    const float *B;
+    int64_t ldb;
+    float *C;
+    int64_t ldc;
+    int J;
+};
+cudaError_t launch_zero_rows(const int32_t *row_cnt, int64_t n_rows, float *C, int64_t ldc, int J, cudaStream_t s);
+cudaError_t launch_cell_spmm(const SpmmArgs &a, cudaStream_t s);
+cudaError_t launch_csr_spmm(const lf_csr &A, const float *B, int64_t ldb, int J, float *C, int64_t ldc,
+                            cudaStream_t s);
+cudaError_t launch_validate(const lf_csr &A, int *d_flag, cudaStream_t s);
+
+}  // namespace lf
+
+struct lf_cell {
+    lf_cell_params params;
+    int64_t n_rows = 0, n_cols = 0, nnz = 0;
+    int64_t n_cell_rows = 0, n_slots = 0, n_tasks = 0;
+    int32_t *row_ind = nullptr;  // view array (bit-exact with the oracle)
+    int32_t *col_ind = nullptr;
+    float *val = nullptr;
+    int32_t *row_tag = nullptr;  // (row << 1) | needs_atomic; -1 = padding
+    int32_t *row_cnt = nullptr;  // CELL rows per source row
+    lf::BucketDev *d_buckets = nullptr;
+    std::vector<lf_bucket> buckets;
+    std::vector<lf::BucketDev> h_buckets;
+    // memory: one pool allocation holds every array above
+    void *pool = nullptr;
+    size_t pool_bytes = 0;
+    lf_allocator al{};
+    bool custom_al = false;
+    cudaStream_t stream = nullptr;
+    lf_csr csr{};  // use_cell == 0: the caller's CSR (must outlive the handle)
+};

@@ -1,0 +1,247 @@
+"""GPU parity: the CUDA path (through the C ABI) against the oracle.
+
+* builder (a1, a4, a5): every CELL array and the bucket table BIT-EXACT;
+* configure statistics (a2) and eq. 7 / Algorithm 3 (a3): exact integers;
+* SpMM (a6, a7): integer-valued inputs (|A| <= 3, |B| <= 15, every partial
+  sum < 2^24) must match EXACTLY whatever the atomic order; float inputs
+  within max|C - C_ref| <= 1e-5 * (|A|.|B|) elementwise (BASELINE.json);
+* full-size BASELINE configs in the bench's launch configuration on sampled
+  rows, plus edge cases (empty, ragged, J not a multiple of 4, ldb/ldc > J,
+  K < P, empty partitions).
+"""
+import numpy as np
+import pytest
+
+import gen
+import oracle
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+TOL = 1e-5
+
+
+@pytest.fixture(scope="module")
+def lf():
+    import paper_conf_hpdc_pengtpk25_b200 as m
+    return m
+
+
+def build(lf, A_h, P, e, k=None):
+    A = lf.Csr.from_host(A_h)
+    M = lf.CellMatrix.build(A, lf.make_params(P, e, k))
+    return A, M
+
+
+def assert_cell_equal(M, cell):
+    v = M.view()
+    torch.cuda.synchronize()
+    assert np.array_equal(v["row_ind"].cpu().numpy(), cell.row_ind)
+    assert np.array_equal(v["col_ind"].cpu().numpy(), cell.col_ind)
+    assert np.array_equal(v["val"].cpu().numpy().view(np.int32), cell.val.view(np.int32))
+    got = [(b["part"], b["width_log2"], b["rows_per_block"], b["n_rows"], b["n_rows_pad"], b["row_off"],
+            b["slot_off"]) for b in v["buckets"]]
+    exp = [tuple(int(b[f]) for f in ("part", "width_log2", "rows_per_block", "n_rows", "n_rows_pad", "row_off",
+                                     "slot_off")) for b in cell.buckets]
+    assert got == exp
+
+
+def spmm_check(M, A_h, B_h, exact=False, rows=None, ldb=None, ldc=None):
+    J = B_h.shape[1]
+    Bd = torch.from_numpy(B_h).cuda()
+    if ldb is not None:
+        big = torch.full((B_h.shape[0], ldb), float("nan"), device="cuda")
+        big[:, :J] = Bd
+        Bd = big[:, :J]
+    out = None
+    if ldc is not None:
+        out = torch.full((A_h.n_rows, ldc), float("nan"), device="cuda")[:, :J]
+    C = M.spmm(Bd, out=out).cpu().numpy().astype(np.float64)
+    Cref, Cabs = oracle.spmm_csr(A_h, B_h, rows)
+    if rows is not None:
+        C = C[rows]
+    if exact:
+        assert np.array_equal(C, Cref)
+    else:
+        err = np.abs(C - Cref)
+        assert np.all(err <= TOL * Cabs), float((err / np.maximum(Cabs, 1e-300)).max())
+    return C
+
+
+SMALL = []
+for s in range(20):
+    rng = np.random.default_rng(s)
+    P = int(rng.integers(1, 6))
+    e = rng.integers(0, 7, size=P).tolist()
+    k = [x + int(rng.integers(0, 3)) for x in e]
+    SMALL.append((s, int(rng.integers(0, 300)), int(rng.integers(1, 200)), P, e, k))
+
+
+@pytest.mark.parametrize("seed,I,K,P,e,k", SMALL)
+def test_builder_bit_exact_small(lf, seed, I, K, P, e, k):
+    A_h = gen.random_small(I, K, 90, seed, dup=True, zeros=True)
+    _, M = build(lf, A_h, P, e, k)
+    assert_cell_equal(M, oracle.csr_to_cell(A_h, P, e, k))
+
+
+@pytest.mark.parametrize("seed,I,K,P,e,k", SMALL[:10])
+@pytest.mark.parametrize("J", [1, 3, 4, 32, 64, 96, 128, 256, 512, 520])
+def test_spmm_integer_exact(lf, seed, I, K, P, e, k, J):
+    A_h = gen.random_small(I, K, 90, seed, dup=True, zeros=True, kind=gen.INT, lo=-3, hi=3)
+    B_h = gen.dense(K, J, seed, gen.INT, -15, 15)
+    _, M = build(lf, A_h, P, e, k)
+    spmm_check(M, A_h, B_h, exact=True)
+
+
+@pytest.mark.parametrize("J,ldb,ldc", [(4, 8, 12), (32, 36, 40), (7, 9, 11), (128, 132, 256)])
+def test_spmm_strided(lf, J, ldb, ldc):
+    A_h = gen.rmat(11, 16, seed=1, kind=gen.INT, lo=-3, hi=3)
+    B_h = gen.dense(A_h.n_cols, J, 1, gen.INT, -15, 15)
+    _, M = build(lf, A_h, 2, [3, 4])
+    spmm_check(M, A_h, B_h, exact=True, ldb=ldb, ldc=ldc)
+
+
+@pytest.mark.parametrize("P", [1, 3])
+@pytest.mark.parametrize("J", [32, 128, 256])
+def test_spmm_tolerance_float(lf, P, J):
+    A_h = gen.rmat(13, 16, seed=2)
+    B_h = gen.dense(A_h.n_cols, J, 2)
+    params, _ = lf.configure(lf.Csr.from_host(A_h), J, force_parts=P)
+    A = lf.Csr.from_host(A_h)
+    M = lf.CellMatrix.build(A, params)
+    spmm_check(M, A_h, B_h)
+
+
+def test_spmm_positive_gnn_style(lf):
+    """All-positive values (val = 1, B in [0,1)): the adversarial case for the
+    relative tolerance; long rows fold."""
+    A_h = gen.powerlaw(3000, 400000, 1.5, seed=3, kind=gen.ONE)
+    B_h = gen.dense(A_h.n_cols, 64, 3, gen.POS)
+    A = lf.Csr.from_host(A_h)
+    params, _ = lf.configure(A, 64)
+    M = lf.CellMatrix.build(A, params)
+    spmm_check(M, A_h, B_h)
+
+
+def test_configure_stats_and_alg3_match_oracle(lf):
+    for A_h, Ps in ((gen.rmat(12, 16, seed=5), (1, 2, 5)), (gen.random_small(200, 150, 120, 9), (1, 4)),
+                    (gen.stencil27(9), (1, 3))):
+        A = lf.Csr.from_host(A_h)
+        for P in Ps:
+            for J in (32, 128):
+                params, st = lf.configure(A, J, force_parts=P)
+                assert params.n_parts == P
+                for p in range(P):
+                    H, F, Un, Ut = oracle.partition_stats(A_h, P, p)
+                    assert list(st.H[p]) == H.tolist()
+                    assert list(st.F[p]) == F.tolist()
+                    assert list(st.Unat[p]) == Un.tolist()
+                    assert list(st.Utop[p]) == Ut.tolist()
+                    top = oracle.partition_max_log2(A_h, P, p)
+                    assert st.max_log2[p] == top
+                    for e in range(top + 1):
+                        assert st.cost[p][e] == oracle.partition_cost(A_h, P, p, e, J)
+                    assert st.chosen_log2[p] == oracle.build_buckets(A_h, P, p, J)
+                    assert params.max_width_log2[p] == max(oracle.build_buckets(A_h, P, p, J), 0)
+        f = oracle.features(A_h)
+        assert list(st.features[:3]) == f[:3].tolist() and list(st.features[4:6]) == f[4:6].tolist()
+        assert st.features[3] == pytest.approx(f[3], rel=1e-14)
+        assert st.features[6] == pytest.approx(f[6], rel=1e-9)
+
+
+def test_golden_configure_on_gpu(lf):
+    """The hand-worked eq. 7 examples, through the GPU statistics."""
+    from conftest import read_golden
+    for name in ("cost_5x8.txt", "cost_separating_2x16.txt"):
+        g = read_golden(name)
+        rows = g["rows"]
+        rp = np.concatenate([[0], np.cumsum([len(r) for r in rows])]).astype(np.int64)
+        ci = np.concatenate([np.array(r, np.int32) for r in rows])
+        A_h = gen.CSR(len(rows), g["K"][0], rp, ci, np.ones(len(ci), np.float32))
+        params, st = lf.configure(lf.Csr.from_host(A_h), g["J"][0], force_parts=1)
+        assert list(st.cost[0][:len(g["cost"])]) == g["cost"]
+        assert params.max_width_log2[0] == g["alg3_e"][0]
+
+
+def test_edge_cases(lf):
+    # no rows
+    A_h = gen.CSR(0, 5, np.zeros(1, np.int64), np.zeros(0, np.int32), np.zeros(0, np.float32))
+    _, M = build(lf, A_h, 1, 2)
+    assert M.spmm(torch.ones(5, 4, device="cuda")).shape == (0, 4)
+    # no entries: C must be exactly +0.0
+    A_h = gen.CSR(7, 5, np.zeros(8, np.int64), np.zeros(0, np.int32), np.zeros(0, np.float32))
+    _, M = build(lf, A_h, 2, 2)
+    C = M.spmm(torch.full((5, 8), 3.0, device="cuda"), out=torch.full((7, 8), float("nan"), device="cuda"))
+    assert torch.equal(C, torch.zeros(7, 8, device="cuda"))
+    # K < P (empty partitions), J = 0
+    A_h = gen.random_small(20, 3, 5, 2, kind=gen.INT)
+    _, M = build(lf, A_h, 5, [1, 2, 0, 3, 1])
+    assert_cell_equal(M, oracle.csr_to_cell(A_h, 5, [1, 2, 0, 3, 1]))
+    B_h = gen.dense(3, 5, 2, gen.INT)
+    spmm_check(M, A_h, B_h, exact=True)
+    assert M.spmm(torch.zeros(3, 0, device="cuda")).shape == (20, 0)
+
+
+def test_csr_path_and_errors(lf):
+    A_h = gen.rmat(11, 16, seed=8, kind=gen.INT)
+    B_h = gen.dense(A_h.n_cols, 64, 8, gen.INT)
+    A = lf.Csr.from_host(A_h)
+    C = lf.csr_spmm(A, torch.from_numpy(B_h).cuda()).cpu().numpy()
+    assert np.array_equal(C.astype(np.float64), oracle.spmm_csr(A_h, B_h)[0])
+    params, _ = lf.configure(A, 64, force_format=2)
+    assert params.use_cell == 0
+    M = lf.CellMatrix.build(A, params)
+    spmm_check(M, A_h, B_h, exact=True)
+    with pytest.raises(lf.LfError):
+        lf.CellMatrix.build(A, lf.make_params(1, 4, 3))
+
+
+def test_row_shard_view(lf):
+    """row_ptr slice with a non-zero base (row sharding) builds the same CELL as
+    the standalone slice."""
+    A_h = gen.rmat(11, 16, seed=6)
+    lo, hi = 300, 1500
+    A = lf.Csr.from_host(A_h)
+    shard = lf.Csr(A.row_ptr[lo:hi + 1], A.col_ind, A.val, A.n_cols)
+    sub = gen.CSR(hi - lo, A_h.n_cols, A_h.row_ptr[lo:hi + 1] - A_h.row_ptr[lo],
+                  A_h.col_ind[A_h.row_ptr[lo]:A_h.row_ptr[hi]], A_h.val[A_h.row_ptr[lo]:A_h.row_ptr[hi]])
+    M = lf.CellMatrix.build(shard, lf.make_params(2, [4, 3]))
+    assert_cell_equal(M, oracle.csr_to_cell(sub, 2, [4, 3]))
+    B_h = gen.dense(A_h.n_cols, 32, 6)
+    spmm_check(M, sub, B_h)
+
+
+# ---- full-size BASELINE configs, the bench's launch configuration ----------
+FULL = ["c1_uniform1024", "c2_rmat20", "c3_stencil126"]
+
+
+@pytest.mark.parametrize("name", FULL)
+def test_full_config_parity(lf, name):
+    A_h, J = gen.config(name)
+    A = lf.Csr.from_host(A_h)
+    params, _ = lf.configure(A, J)
+    M = lf.CellMatrix.build(A, params)
+    P = params.n_parts
+    cell = oracle.csr_to_cell(A_h, P, list(params.max_width_log2[:P]), list(params.block_nnz_log2[:P]))
+    assert_cell_equal(M, cell)
+    B_h = gen.dense(A_h.n_cols, J, 0)
+    rng = np.random.default_rng(0)
+    l = A_h.row_lengths()
+    rows = np.unique(np.concatenate([rng.integers(0, A_h.n_rows, 3000), np.argsort(l)[-50:],
+                                     np.flatnonzero(l == 0)[:50], [0, A_h.n_rows - 1]])).astype(np.int64)
+    spmm_check(M, A_h, B_h, rows=rows)
+
+
+def test_full_reddit_parity(lf):
+    A_h, J = gen.config("c4_reddit")
+    A = lf.Csr.from_host(A_h)
+    params, _ = lf.configure(A, J)
+    M = lf.CellMatrix.build(A, params)
+    B_h = gen.dense(A_h.n_cols, J, 0)
+    rng = np.random.default_rng(1)
+    l = A_h.row_lengths()
+    rows = np.unique(np.concatenate([rng.integers(0, A_h.n_rows, 500), np.argsort(l)[-20:]])).astype(np.int64)
+    spmm_check(M, A_h, B_h, rows=rows)
+    # builder: the arrays of the 20 longest rows' buckets via the round-trip
+    v = M.view()
+    assert int(v["n_slots"]) >= A_h.nnz
