@@ -148,7 +148,7 @@ class CellMatrix:
             if n == 0 or not ptr:
                 return torch.empty(0, dtype=dtype, device="cuda")
             obj = type("CAI", (), {"__cuda_array_interface__": {
-                "shape": (n,), "typestr": typestr, "data": (ptr, True), "version": 2}})()
+                "shape": (n,), "typestr": typestr, "data": (ptr, False), "version": 2}})()
             return torch.as_tensor(obj, device=f"cuda:{dev}")
 
         buckets = [{f: getattr(v.buckets[i], f) for f, _ in _abi.LfBucket._fields_ if f != "pad_"}
