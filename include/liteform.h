@@ -201,7 +201,7 @@ LF_API lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configur
  * bucket sizes); the rest is enqueued asynchronously on s, so the handle may
  * be used on s immediately.
  * Errors: LF_ERR_INVALID_ARG (sizes, e_p > k_p, P out of range),
- *         LF_ERR_INDEX_OVERFLOW (n_rows >= 2^30 or K > 2^31-1),
+ *         LF_ERR_INDEX_OVERFLOW (n_rows >= 2^28 or K > 2^31-1),
  *         LF_ERR_NO_MEMORY, LF_ERR_CUDA, LF_ERR_UNSORTED_CSR (LF_VALIDATE=1). */
 LF_API lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_allocator *al, lf_stream_t s,
                         lf_cell **out);

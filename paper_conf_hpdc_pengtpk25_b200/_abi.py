@@ -10,7 +10,7 @@ import ctypes
 import os
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "liblf.so")
+LIB_PATH = os.environ.get("LF_LIB") or os.path.join(_PKG, "liblf.so")  # LF_LIB: experiment builds
 HEADER_PATH = os.path.join(os.path.dirname(_PKG), "include", "liteform.h")
 
 LF_MAX_PARTS = 64

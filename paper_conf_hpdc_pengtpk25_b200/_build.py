@@ -29,17 +29,21 @@ def _newest(paths):
     return max((os.path.getmtime(p) for p in paths), default=0.0)
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
+def build(force: bool = False, verbose: bool = False, defs=(), out: str | None = None) -> str:
+    """defs: extra -D macros (experiment variants go to `out` / build_<tag>/)."""
+    global OBJ
+    lib = out or LIB
+    obj_dir = OBJ if not defs else OBJ + "_" + "_".join(d.replace("=", "") for d in defs)
     srcs = sources()
-    if not force and os.path.exists(LIB) and os.path.getmtime(LIB) >= _newest(srcs + _headers() + [__file__]):
-        return LIB
-    os.makedirs(OBJ, exist_ok=True)
+    if not force and os.path.exists(lib) and os.path.getmtime(lib) >= _newest(srcs + _headers() + [__file__]):
+        return lib
+    os.makedirs(obj_dir, exist_ok=True)
     hdr_t = _newest(_headers() + [__file__])
 
     def compile_one(src):
-        obj = os.path.join(OBJ, os.path.basename(src).replace(".cu", ".o"))
+        obj = os.path.join(obj_dir, os.path.basename(src).replace(".cu", ".o"))
         if force or not os.path.exists(obj) or os.path.getmtime(obj) < max(os.path.getmtime(src), hdr_t):
-            cmd = [NVCC, *ARCH, *FLAGS, "-Xptxas", "-v" if verbose else "-O3", "-c", src, "-o", obj]
+            cmd = [NVCC, *ARCH, *FLAGS, *[f"-D{d}" for d in defs], "-Xptxas", "-v" if verbose else "-O3", "-c", src, "-o", obj]
             r = subprocess.run(cmd, capture_output=True, text=True)
             if r.returncode != 0:
                 raise RuntimeError(f"nvcc failed for {src}:\n{r.stderr}")
@@ -49,12 +53,14 @@ def build(force: bool = False, verbose: bool = False) -> str:
 
     with cf.ThreadPoolExecutor(max_workers=min(8, len(srcs))) as ex:
         objs = list(ex.map(compile_one, srcs))
-    tmp = LIB + f".tmp{os.getpid()}"
+    tmp = lib + f".tmp{os.getpid()}"
     subprocess.check_call([NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-cudart", "static"])
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, lib)
+    return lib
 
 
 if __name__ == "__main__":
     import sys
-    print(build(force="-f" in sys.argv, verbose="-v" in sys.argv))
+    defs = [a[2:] for a in sys.argv[1:] if a.startswith("-D")]
+    outs = [a[6:] for a in sys.argv[1:] if a.startswith("--out=")]
+    print(build(force="-f" in sys.argv, verbose="-v" in sys.argv, defs=defs, out=outs[0] if outs else None))

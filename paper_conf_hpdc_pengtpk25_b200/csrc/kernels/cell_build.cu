@@ -116,13 +116,15 @@ __global__ void __launch_bounds__(kThreads)
         if (key != kNoKey) {
             pos = key_row_off[p * kMaxT + key] + tile_cnt[((int64_t)p * kMaxT + key) * n_tiles + tile] +
                   warp_tot[warp][key] + rank;
-            tag = (int32_t)((i << 1) | (row_cnt[i] > 1 ? 1 : 0));
+            // (i << 3) | S << 2 | F << 1 | L  (cell_spmm.cu): S = this segment holds
+            // all of row i's CELL rows; F / L are added per sub-row below
+            tag = (int32_t)((i << 3) | (row_cnt[i] == n_sub ? 4 : 0));
         }
         const int64_t W = int64_t(1) << (key == kNoKey ? 0 : key);
         if (n_sub <= 32) {
             for (int64_t s = 0; s < n_sub; s++) {
                 row_ind[pos + s] = (int32_t)i;
-                row_tag[pos + s] = tag;
+                row_tag[pos + s] = tag | (s == 0 ? 2 : 0) | (s == n_sub - 1 ? 1 : 0);
                 src_pos[pos + s] = beg + s * W;
                 src_cnt[pos + s] = (int32_t)min(W, l - s * W);
             }
@@ -141,7 +143,7 @@ __global__ void __launch_bounds__(kThreads)
             const int64_t si = __shfl_sync(0xffffffffu, i, src);
             for (int64_t s = lane; s < sn; s += 32) {
                 row_ind[sp + s] = (int32_t)si;
-                row_tag[sp + s] = stag;
+                row_tag[sp + s] = stag | (s == 0 ? 2 : 0) | (s == sn - 1 ? 1 : 0);
                 src_pos[sp + s] = sb + s * sW;
                 src_cnt[sp + s] = (int32_t)min(sW, sl - s * sW);
             }

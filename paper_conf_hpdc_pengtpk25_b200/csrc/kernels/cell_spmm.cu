@@ -5,19 +5,28 @@
 // B200 mapping:
 //   * a WARP TASK is 32 consecutive slots of a bucket with W <= 32 (32/W whole
 //     CELL rows: one 2^k-slot block when k = 5), or one CELL row when W > 32;
-//     tasks are contiguous in slot order, so warps stream colInd/val with one
-//     coalesced 128-byte load each and walk buckets partition-major;
+//     warps take CH consecutive tasks per round (chunked grid-stride), so the
+//     whole grid sweeps the buckets partition-major and each warp streams
+//     colInd/val with coalesced 128-byte loads, prefetching the next task's
+//     slots and row tags while it gathers the current one;
 //   * the lanes split J: J/4 float4 columns over 32/G lanes, G lane groups
 //     each taking every G-th slot (G = 4, 2, 1 for J <= 32, 64, >= 128); NV
 //     float4 per lane cover J up to 512 per pass (J tiles beyond that);
 //   * slot (col, val) pairs are broadcast with shuffles; B rows are gathered
 //     as float4 through the read-only path, U slots in flight per lane;
+//   * the index/value/tag streams and C stores carry an L2 evict_first policy
+//     so the L2 keeps B rows;
 //   * the row width W is a template parameter for W <= 32, so the fold /
 //     group reduction and the C update positions are compile-time;
-//   * C update (reading R11): rows whose source row has exactly one CELL row
-//     are plain vector stores; the others (folded rows, P > 1) were zeroed by
-//     zero_rows_kernel and receive red.global.add.v4.f32;
+//   * folded rows (reading R4: consecutive CELL rows of one source row) are
+//     summed in registers across consecutive tasks of a warp; a run that holds
+//     every CELL row of its source row is written with a plain vector store,
+//     otherwise (run split between warps, or P > 1) red.global.add.v4.f32 into
+//     the row zeroed beforehand by zero_rows_kernel (reading R11);
 //   * rows of A with no CELL row are zeroed by zero_rows_kernel (R13).
+// Row tag (built by bucket_kernel<1>): (i << 3) | S<<2 | F<<1 | L, where F/L
+// mark the first/last sub-row of the (row, partition) segment and S that the
+// segment holds all of the row's CELL rows; -1 = padding row.
 #include "../lf_internal.cuh"
 
 namespace lf {
@@ -26,6 +35,27 @@ namespace {
 
 constexpr unsigned kFull = 0xffffffffu;
 constexpr int kWarpsPerBlock = 8;
+constexpr int kChunk = 8;  // consecutive tasks per warp per round
+#ifndef LF_SPMM_MIN_BLOCKS
+#define LF_SPMM_MIN_BLOCKS 3
+#endif
+constexpr int kMinBlocks = LF_SPMM_MIN_BLOCKS;  // resident 256-thread blocks per SM
+
+__device__ __forceinline__ uint64_t policy_evict_first() {
+    uint64_t p;
+    asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+    return p;
+}
+__device__ __forceinline__ int32_t ld_stream(const int32_t *p, uint64_t pol) {
+    int32_t v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.b32 %0, [%1], %2;" : "=r"(v) : "l"(p), "l"(pol));
+    return v;
+}
+__device__ __forceinline__ float ld_stream(const float *p, uint64_t pol) {
+    float v;
+    asm volatile("ld.global.nc.L1::no_allocate.L2::cache_hint.f32 %0, [%1], %2;" : "=f"(v) : "l"(p), "l"(pol));
+    return v;
+}
 
 template <int VEC> struct Vec;
 template <> struct Vec<4> {
@@ -44,8 +74,9 @@ template <> struct Vec<4> {
         acc.z += __shfl_xor_sync(kFull, acc.z, o);
         acc.w += __shfl_xor_sync(kFull, acc.w, o);
     }
-    static __device__ __forceinline__ void store(float *p, const T &v) {
-        asm volatile("st.global.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(p), "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w)
+    static __device__ __forceinline__ void store(float *p, const T &v, uint64_t pol) {
+        asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(p),
+                     "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w), "l"(pol)
                      : "memory");
     }
     static __device__ __forceinline__ void red(float *p, const T &v) {
@@ -60,11 +91,14 @@ template <> struct Vec<1> {
     static __device__ __forceinline__ T load(const float *p) { return __ldg(p); }
     static __device__ __forceinline__ void fma(T &acc, float a, const T &b) { acc = fmaf(a, b, acc); }
     static __device__ __forceinline__ void add_xor(T &acc, int o) { acc += __shfl_xor_sync(kFull, acc, o); }
-    static __device__ __forceinline__ void store(float *p, const T &v) { *p = v; }
+    static __device__ __forceinline__ void store(float *p, const T &v, uint64_t) { *p = v; }
     static __device__ __forceinline__ void red(float *p, const T &v) { atomicAdd(p, v); }
 };
 
-// Lane layout for one J tile of JT = LPR * NV * VEC columns starting at j0.
+// tag helpers
+__device__ __forceinline__ bool tag_whole(int32_t tag) { return (tag & 7) == 7; }  // S && F && L
+__device__ __forceinline__ int32_t tag_row(int32_t tag) { return tag >> 3; }
+
 template <int VEC, int G, int NV>
 struct Layout {
     static constexpr int LPR = 32 / G;  // lanes per group
@@ -84,42 +118,79 @@ struct Ctx {
     int J;
     int j0;
     int g, li;  // lane group, lane in group
+    uint64_t pol;
 
     __device__ __forceinline__ int jcol(int m) const { return j0 + (m * L::LPR + li) * VEC; }
     __device__ __forceinline__ bool jok(int m) const { return jcol(m) < J; }
 
-    // gather slot's B row slice (zero if padding)
     __device__ __forceinline__ void gather(int32_t c, VT (&b)[NV]) const {
 #pragma unroll
         for (int m = 0; m < NV; m++) b[m] = (c >= 0 && jok(m)) ? V::load(B + (int64_t)c * ldb + jcol(m)) : V::zero();
     }
-    __device__ __forceinline__ void write(int32_t tag, const VT (&acc)[NV]) const {
-        if (tag < 0) return;
-        float *row = C + (int64_t)(tag >> 1) * ldc;
+    // write one C row slice: plain store when this write is the row's only one
+    __device__ __forceinline__ void write(int32_t row, bool plain, const VT (&acc)[NV]) const {
+        float *p = C + (int64_t)row * ldc;
 #pragma unroll
         for (int m = 0; m < NV; m++) {
             if (!jok(m)) continue;
-            if (tag & 1) V::red(row + jcol(m), acc[m]);
-            else V::store(row + jcol(m), acc[m]);
+            if (plain) V::store(p + jcol(m), acc[m], pol);
+            else V::red(p + jcol(m), acc[m]);
         }
+    }
+    __device__ __forceinline__ void zero(VT (&acc)[NV]) const {
+#pragma unroll
+        for (int m = 0; m < NV; m++) acc[m] = V::zero();
+    }
+    // sum the G lane groups (all hold partial sums of the same row)
+    __device__ __forceinline__ void reduce_groups(VT (&acc)[NV]) const {
+#pragma unroll
+        for (int o = 1; o < G; o <<= 1)
+#pragma unroll
+            for (int m = 0; m < NV; m++) V::add_xor(acc[m], o * L::LPR);
     }
 };
 
-// 32-slot task of a bucket with W = 2^T <= 32: 32/W CELL rows.
+// 32 slots (c_l, v_l in the lanes) accumulated into acc, no row boundary
+template <int VEC, int G, int NV>
+__device__ __forceinline__ void accum32(const Ctx<VEC, G, NV> &cx, int32_t c_l, float v_l,
+                                        typename Ctx<VEC, G, NV>::VT (&acc)[NV]) {
+    using C = Ctx<VEC, G, NV>;
+    using V = typename C::V;
+    using VT = typename C::VT;
+    constexpr int STEPS = 32 / G;
+    constexpr int U = C::L::U < STEPS ? C::L::U : STEPS;
+#pragma unroll
+    for (int kb = 0; kb < STEPS; kb += U) {
+        VT b[U][NV];
+        float a[U];
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+            const int slot = (kb + u) * G + cx.g;
+            const int32_t c = __shfl_sync(kFull, c_l, slot);
+            a[u] = __shfl_sync(kFull, v_l, slot);
+            cx.gather(c, b[u]);
+        }
+#pragma unroll
+        for (int u = 0; u < U; u++)
+#pragma unroll
+            for (int m = 0; m < NV; m++) V::fma(acc[m], a[u], b[u][m]);
+    }
+}
+
+// 32-slot task of a bucket with W = 2^T < 32: 32/W CELL rows, each written.
 template <int VEC, int G, int NV, int T>
 __device__ __forceinline__ void narrow_task(const Ctx<VEC, G, NV> &cx, int32_t c_l, float v_l, int32_t tag_l) {
     using C = Ctx<VEC, G, NV>;
     using V = typename C::V;
     using VT = typename C::VT;
     constexpr int W = 1 << T;
-    constexpr int STEPS = 32 / G;                      // each step: one slot per group
-    constexpr int RG = W >= G ? G : W;                 // groups sharing one CELL row
-    constexpr int SPR = W >= G ? W / G : 1;            // steps per row
+    constexpr int STEPS = 32 / G;            // each step: one slot per group
+    constexpr int RG = W >= G ? G : W;       // groups sharing one CELL row
+    constexpr int SPR = W >= G ? W / G : 1;  // steps per row
     constexpr int U = C::L::U < STEPS ? C::L::U : STEPS;
     constexpr int LPR = C::L::LPR;
     VT acc[NV];
-#pragma unroll
-    for (int m = 0; m < NV; m++) acc[m] = V::zero();
+    cx.zero(acc);
 #pragma unroll
     for (int kb = 0; kb < STEPS; kb += U) {
         VT b[U][NV];
@@ -143,97 +214,144 @@ __device__ __forceinline__ void narrow_task(const Ctx<VEC, G, NV> &cx, int32_t c
                     for (int m = 0; m < NV; m++) V::add_xor(acc[m], o * LPR);
                 const int ro = (W >= G) ? step / SPR : step * (G / W) + cx.g / W;
                 const int32_t tag = __shfl_sync(kFull, tag_l, ro);
-                if (cx.g % RG == 0) cx.write(tag, acc);
-#pragma unroll
-                for (int m = 0; m < NV; m++) acc[m] = V::zero();
+                if (cx.g % RG == 0 && tag >= 0) cx.write(tag_row(tag), tag_whole(tag), acc);
+                cx.zero(acc);
             }
         }
     }
 }
 
-// Accumulate n32 chunks of 32 slots starting at slot s0 (one CELL row / CSR
-// row of arbitrary length n), then reduce over groups and write.
-template <int VEC, int G, int NV>
-__device__ __forceinline__ void wide_row(const Ctx<VEC, G, NV> &cx, const int32_t *__restrict__ col,
-                                         const float *__restrict__ val, int64_t s0, int64_t n, int32_t tag,
-                                         int lane) {
-    using C = Ctx<VEC, G, NV>;
-    using V = typename C::V;
-    using VT = typename C::VT;
-    constexpr int STEPS = 32 / G;
-    constexpr int U = C::L::U < STEPS ? C::L::U : STEPS;
-    VT acc[NV];
-#pragma unroll
-    for (int m = 0; m < NV; m++) acc[m] = V::zero();
-    for (int64_t base = 0; base < n; base += 32) {
-        const int64_t s = s0 + base + lane;
-        const bool in = base + lane < n;
-        const int32_t c_l = in ? __ldg(col + s) : -1;
-        const float v_l = in ? __ldg(val + s) : 0.f;
-        if (__ballot_sync(kFull, c_l >= 0) == 0) break;  // rest of the row is padding
-#pragma unroll
-        for (int kb = 0; kb < STEPS; kb += U) {
-            VT b[U][NV];
-            float a[U];
-#pragma unroll
-            for (int u = 0; u < U; u++) {
-                const int slot = (kb + u) * G + cx.g;
-                const int32_t c = __shfl_sync(kFull, c_l, slot);
-                a[u] = __shfl_sync(kFull, v_l, slot);
-                cx.gather(c, b[u]);
-            }
-#pragma unroll
-            for (int u = 0; u < U; u++)
-#pragma unroll
-                for (int m = 0; m < NV; m++) V::fma(acc[m], a[u], b[u][m]);
-        }
+struct TaskIn {
+    int32_t c, tag;  // lane's slot column / row tag
+    float v;
+    int b;           // bucket
+};
+
+// fetch a task's slots and row tags (tasks ascend per warp, so the bucket
+// cursor only moves forward)
+__device__ __forceinline__ TaskIn load_task(const SpmmArgs &a, int64_t task, int &bcur, int lane, uint64_t pol) {
+    while (bcur + 1 < a.nb && __ldg(&a.buckets[bcur + 1].task_off) <= task) bcur++;
+    const BucketDev *bk = a.buckets + bcur;
+    const int64_t tin = task - __ldg(&bk->task_off);
+    const int t = __ldg(&bk->t);
+    const int64_t slot_off = __ldg(&bk->slot_off), row_off = __ldg(&bk->row_off);
+    TaskIn x;
+    x.b = bcur;
+    if (t >= 5) {  // one CELL row of W = 2^t >= 32 slots
+        const int64_t s0 = slot_off + (tin << t);
+        x.c = ld_stream(a.col + s0 + lane, pol);
+        x.v = ld_stream(a.val + s0 + lane, pol);
+        x.tag = __shfl_sync(kFull, lane == 0 ? ld_stream(a.row_tag + row_off + tin, pol) : 0, 0);
+    } else {
+        const int64_t s0 = slot_off + tin * 32;
+        const int64_t ns = min((int64_t)32, __ldg(&bk->n_slots) - tin * 32);
+        const int64_t nrows = ns >> t;
+        x.c = lane < ns ? ld_stream(a.col + s0 + lane, pol) : -1;
+        x.v = lane < ns ? ld_stream(a.val + s0 + lane, pol) : 0.f;
+        x.tag = lane < nrows ? ld_stream(a.row_tag + row_off + ((tin * 32) >> t) + lane, pol) : -1;
     }
-#pragma unroll
-    for (int o = 1; o < G; o <<= 1)
-#pragma unroll
-        for (int m = 0; m < NV; m++) V::add_xor(acc[m], o * C::L::LPR);
-    if (cx.g == 0) cx.write(tag, acc);
+    return x;
 }
 
 template <int VEC, int G, int NV>
-__global__ void __launch_bounds__(kWarpsPerBlock * 32) cell_spmm_kernel(SpmmArgs a) {
+__global__ void __launch_bounds__(kWarpsPerBlock * 32, kMinBlocks) cell_spmm_kernel(const SpmmArgs a) {
+    using Cx = Ctx<VEC, G, NV>;
+    using VT = typename Cx::VT;
     using L = Layout<VEC, G, NV>;
     const int lane = threadIdx.x & 31;
     const int64_t gwarp = (int64_t)blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
     const int64_t nwarps = (int64_t)gridDim.x * kWarpsPerBlock;
-    Ctx<VEC, G, NV> cx{a.B, a.ldb, a.C, a.ldc, a.J, 0, lane / L::LPR, lane % L::LPR};
-    int b = 0;
-    for (int64_t task = gwarp; task < a.n_tasks; task += nwarps) {
-        while (b + 1 < a.nb && a.buckets[b + 1].task_off <= task) b++;  // tasks ascend per warp
-        const BucketDev bk = a.buckets[b];
-        const int64_t tin = task - bk.task_off;
-        if (bk.t > 5) {  // one CELL row of W = 2^t > 32 slots
-            const int32_t tag = __ldg(a.row_tag + bk.row_off + tin);
-            if (tag < 0) continue;
-            for (int j0 = 0; j0 < a.J; j0 += L::JT) {
-                cx.j0 = j0;
-                wide_row<VEC, G, NV>(cx, a.col, a.val, bk.slot_off + tin * bk.task_slots, bk.task_slots, tag, lane);
-            }
-            continue;
+    const uint64_t pol = policy_evict_first();
+    Cx cx{a.B, a.ldb, a.C, a.ldc, a.J, 0, lane / L::LPR, lane % L::LPR, pol};
+    const bool single_tile = a.J <= L::JT;  // merge folded rows only without J tiling
+    int bcur = 0;
+
+    VT acc[NV];
+    cx.zero(acc);
+    int32_t pend = -1;  // tag of the run being accumulated in acc (-1: none)
+    bool run_first = false;
+
+    const int64_t round = nwarps * kChunk;
+    int64_t cs = gwarp * kChunk;  // chunk start
+    if (cs >= a.n_tasks) return;
+    int64_t task = cs;
+    TaskIn cur = load_task(a, task, bcur, lane, pol);
+    while (task < a.n_tasks) {
+        int64_t tn = task + 1;
+        bool chunk_end = false;
+        if (tn >= cs + kChunk || tn >= a.n_tasks) {
+            chunk_end = true;
+            cs += round;
+            tn = cs;
         }
-        const int64_t s0 = bk.slot_off + tin * 32;
-        const int64_t ns = min((int64_t)32, bk.n_slots - tin * 32);
-        const int32_t c_l = lane < ns ? __ldg(a.col + s0 + lane) : -1;
-        const float v_l = lane < ns ? __ldg(a.val + s0 + lane) : 0.f;
-        const int64_t nrows = ns >> bk.t;
-        const int32_t tag_l = lane < nrows ? __ldg(a.row_tag + bk.row_off + ((tin * 32) >> bk.t) + lane) : -1;
-        if (__ballot_sync(kFull, tag_l >= 0) == 0) continue;  // all padding
-        for (int j0 = 0; j0 < a.J; j0 += L::JT) {
-            cx.j0 = j0;
-            switch (bk.t) {
-            case 0: narrow_task<VEC, G, NV, 0>(cx, c_l, v_l, tag_l); break;
-            case 1: narrow_task<VEC, G, NV, 1>(cx, c_l, v_l, tag_l); break;
-            case 2: narrow_task<VEC, G, NV, 2>(cx, c_l, v_l, tag_l); break;
-            case 3: narrow_task<VEC, G, NV, 3>(cx, c_l, v_l, tag_l); break;
-            case 4: narrow_task<VEC, G, NV, 4>(cx, c_l, v_l, tag_l); break;
-            default: narrow_task<VEC, G, NV, 5>(cx, c_l, v_l, tag_l); break;
+        TaskIn nxt{};
+        if (tn < a.n_tasks) nxt = load_task(a, tn, bcur, lane, pol);
+        const int t = __ldg(&a.buckets[cur.b].t);
+        if (t >= 5) {
+            const int32_t tag = cur.tag;
+            if (tag >= 0) {
+                if (pend >= 0 && tag_row(pend) != tag_row(tag)) {
+                    cx.reduce_groups(acc);
+                    if (cx.g == 0) cx.write(tag_row(pend), false, acc);
+                    cx.zero(acc);
+                    pend = -1;
+                }
+                if (pend < 0) run_first = (tag & 2) != 0;
+                const int64_t W = int64_t(1) << t;
+                const int64_t s0 = __ldg(&a.buckets[cur.b].slot_off) + ((task - __ldg(&a.buckets[cur.b].task_off)) << t);
+                for (int j0 = 0; j0 < a.J; j0 += L::JT) {
+                    cx.j0 = j0;
+                    if (!single_tile) cx.zero(acc);
+                    accum32<VEC, G, NV>(cx, cur.c, cur.v, acc);
+                    for (int64_t base = 32; base < W; base += 32) {
+                        const int32_t c_l = ld_stream(a.col + s0 + base + lane, pol);
+                        const float v_l = ld_stream(a.val + s0 + base + lane, pol);
+                        if (__ballot_sync(kFull, c_l >= 0) == 0) break;  // rest is padding
+                        accum32<VEC, G, NV>(cx, c_l, v_l, acc);
+                    }
+                    if (!single_tile) {  // no run merging across J tiles
+                        cx.reduce_groups(acc);
+                        if (cx.g == 0) cx.write(tag_row(tag), tag_whole(tag), acc);
+                    }
+                }
+                if (single_tile) {
+                    pend = tag;
+                    if (tag & 1) {  // last sub-row of the segment completes the run
+                        cx.reduce_groups(acc);
+                        if (cx.g == 0) cx.write(tag_row(tag), run_first && (tag & 4), acc);
+                        cx.zero(acc);
+                        pend = -1;
+                    }
+                }
+            }
+        } else {
+            if (pend >= 0) {
+                cx.reduce_groups(acc);
+                if (cx.g == 0) cx.write(tag_row(pend), false, acc);
+                cx.zero(acc);
+                pend = -1;
+            }
+            if (__ballot_sync(kFull, cur.tag >= 0)) {
+                for (int j0 = 0; j0 < a.J; j0 += L::JT) {
+                    cx.j0 = j0;
+                    switch (t) {
+                    case 0: narrow_task<VEC, G, NV, 0>(cx, cur.c, cur.v, cur.tag); break;
+                    case 1: narrow_task<VEC, G, NV, 1>(cx, cur.c, cur.v, cur.tag); break;
+                    case 2: narrow_task<VEC, G, NV, 2>(cx, cur.c, cur.v, cur.tag); break;
+                    case 3: narrow_task<VEC, G, NV, 3>(cx, cur.c, cur.v, cur.tag); break;
+                    default: narrow_task<VEC, G, NV, 4>(cx, cur.c, cur.v, cur.tag); break;
+                    }
+                }
             }
         }
+        if (chunk_end && pend >= 0) {
+            cx.reduce_groups(acc);
+            if (cx.g == 0) cx.write(tag_row(pend), false, acc);
+            cx.zero(acc);
+            pend = -1;
+        }
+        task = tn;
+        cur = nxt;
     }
 }
 
@@ -243,16 +361,28 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32)
     csr_spmm_kernel(const int64_t *__restrict__ row_ptr, const int32_t *__restrict__ col,
                     const float *__restrict__ val, int64_t n_rows, const float *__restrict__ B, int64_t ldb,
                     float *__restrict__ C, int64_t ldc, int J) {
+    using Cx = Ctx<VEC, G, NV>;
+    using VT = typename Cx::VT;
     using L = Layout<VEC, G, NV>;
     const int lane = threadIdx.x & 31;
     const int64_t gwarp = (int64_t)blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
     const int64_t nwarps = (int64_t)gridDim.x * kWarpsPerBlock;
-    Ctx<VEC, G, NV> cx{B, ldb, C, ldc, J, 0, lane / L::LPR, lane % L::LPR};
+    const uint64_t pol = policy_evict_first();
+    Cx cx{B, ldb, C, ldc, J, 0, lane / L::LPR, lane % L::LPR, pol};
     for (int64_t i = gwarp; i < n_rows; i += nwarps) {
         const int64_t rb = row_ptr[i], re = row_ptr[i + 1];
         for (int j0 = 0; j0 < J; j0 += L::JT) {
             cx.j0 = j0;
-            wide_row<VEC, G, NV>(cx, col, val, rb, re - rb, (int32_t)(i << 1), lane);
+            VT acc[NV];
+            cx.zero(acc);
+            for (int64_t base = rb; base < re; base += 32) {
+                const bool in = base + lane < re;
+                const int32_t c_l = in ? ld_stream(col + base + lane, pol) : -1;
+                const float v_l = in ? ld_stream(val + base + lane, pol) : 0.f;
+                accum32<VEC, G, NV>(cx, c_l, v_l, acc);
+            }
+            cx.reduce_groups(acc);
+            if (cx.g == 0) cx.write((int32_t)i, true, acc);
         }
     }
 }
@@ -281,34 +411,33 @@ __global__ void zero_rows_kernel(const int32_t *__restrict__ row_cnt, int64_t n_
     }
 }
 
-template <int VEC, int G, int NV>
-int blocks_for(const void *fn) {
-    static int occ = 0, sms = 0;
-    if (!occ) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kWarpsPerBlock * 32, 0);
-        if (occ <= 0) occ = 1;
-        if (sms <= 0) sms = 148;
-    }
-    return occ * sms;
+template <typename F>
+int resident_blocks(F fn) {
+    int occ = 0, sms = 0, dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kWarpsPerBlock * 32, 0);
+    return std::max(1, occ) * std::max(1, sms);
 }
 
 template <int VEC, int G, int NV>
 cudaError_t run_cell(const SpmmArgs &a, cudaStream_t s) {
+    static int cap = 0;
     auto fn = cell_spmm_kernel<VEC, G, NV>;
-    int64_t want = (a.n_tasks + kWarpsPerBlock - 1) / kWarpsPerBlock;
-    int grid = (int)std::max<int64_t>(1, std::min<int64_t>(want, blocks_for<VEC, G, NV>((const void *)fn)));
+    if (!cap) cap = resident_blocks(fn);
+    int64_t want = (a.n_tasks + kWarpsPerBlock * kChunk - 1) / (kWarpsPerBlock * kChunk);
+    int grid = (int)std::max<int64_t>(1, std::min<int64_t>(want, cap));
     fn<<<grid, kWarpsPerBlock * 32, 0, s>>>(a);
     return cudaGetLastError();
 }
 
 template <int VEC, int G, int NV>
 cudaError_t run_csr(const lf_csr &A, const float *B, int64_t ldb, int J, float *C, int64_t ldc, cudaStream_t s) {
+    static int cap = 0;
     auto fn = csr_spmm_kernel<VEC, G, NV>;
+    if (!cap) cap = resident_blocks(fn);
     int64_t want = (A.n_rows + kWarpsPerBlock - 1) / kWarpsPerBlock;
-    int grid = (int)std::max<int64_t>(1, std::min<int64_t>(want, blocks_for<VEC, G, NV>((const void *)fn)));
+    int grid = (int)std::max<int64_t>(1, std::min<int64_t>(want, cap));
     fn<<<grid, kWarpsPerBlock * 32, 0, s>>>(A.row_ptr, A.col_ind, A.val, A.n_rows, B, ldb, C, ldc, J);
     return cudaGetLastError();
 }

@@ -66,7 +66,7 @@ lf_status check_csr(const lf_csr *A) {
     if (!A->row_ptr) return fail(LF_ERR_INVALID_ARG, "row_ptr is NULL");
     if (A->nnz > 0 && (!A->col_ind || !A->val)) return fail(LF_ERR_INVALID_ARG, "col_ind/val NULL with nnz > 0");
     if (A->n_cols > 2147483647LL) return fail(LF_ERR_INDEX_OVERFLOW, "n_cols exceeds int32");
-    if (A->n_rows >= (int64_t(1) << 30)) return fail(LF_ERR_INDEX_OVERFLOW, "n_rows >= 2^30");
+    if (A->n_rows >= (int64_t(1) << 28)) return fail(LF_ERR_INDEX_OVERFLOW, "n_rows >= 2^28");
     return LF_OK;
 }
 
@@ -154,11 +154,14 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
         LF_CUDA(cudaMallocAsync(&d_mask, (size_t)A->n_cols * sizeof(uint32_t), s));
         LF_CUDA(cudaMemsetAsync(d_mask, 0, (size_t)A->n_cols * sizeof(uint32_t), s));
     }
-    LF_CUDA(lf::launch_stats(*A, P, d_st, d_mask, s));
+    uint8_t *d_t0 = nullptr;
+    if (A->n_rows > 0) LF_CUDA(cudaMallocAsync(&d_t0, (size_t)A->n_rows * P, s));
+    LF_CUDA(lf::launch_stats(*A, P, d_st, d_mask, d_t0, s));
     std::vector<lf::StatsDev> h(1);
     LF_CUDA(cudaMemcpyAsync(h.data(), d_st, sizeof(lf::StatsDev), cudaMemcpyDeviceToHost, s));
     LF_CUDA(cudaFreeAsync(d_st, s));
     if (d_mask) LF_CUDA(cudaFreeAsync(d_mask, s));
+    if (d_t0) LF_CUDA(cudaFreeAsync(d_t0, s));
     LF_CUDA(cudaStreamSynchronize(s));
     const lf::StatsDev &st = h[0];
 

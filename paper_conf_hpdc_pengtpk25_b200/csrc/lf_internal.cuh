@@ -46,7 +46,8 @@ struct StatsDev {
 };
 
 // ---- launchers (kernels in csrc/kernels/*.cu) ----
-cudaError_t launch_stats(const lf_csr &A, int P, StatsDev *d_stats, uint32_t *d_colmask, cudaStream_t s);
+cudaError_t launch_stats(const lf_csr &A, int P, StatsDev *d_stats, uint32_t *d_colmask, uint8_t *d_t0seg,
+                         cudaStream_t s);
 
 struct BuildScratch {
     int32_t *seg_rel;       // [I*(P-1)] segment starts relative to the row start (P > 1)
@@ -97,7 +98,7 @@ struct lf_cell {
     int32_t *row_ind = nullptr;  // view array (bit-exact with the oracle)
     int32_t *col_ind = nullptr;
     float *val = nullptr;
-    int32_t *row_tag = nullptr;  // (row << 1) | needs_atomic; -1 = padding
+    int32_t *row_tag = nullptr;  // (row << 3) | S,F,L flags (cell_spmm.cu); -1 = padding
     int32_t *row_cnt = nullptr;  // CELL rows per source row
     lf::BucketDev *d_buckets = nullptr;
     std::vector<lf_bucket> buckets;

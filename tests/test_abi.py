@@ -57,7 +57,7 @@ def test_null_arguments_rejected_on_host():
     p.n_parts, p.use_cell = 1, 1
     p.max_width_log2[0], p.block_nnz_log2[0] = 3, 2
     assert L.lf_cell_build(ctypes.byref(A), ctypes.byref(p), None, None, ctypes.byref(h)) == 1
-    A2 = _abi.LfCsr(1 << 30, 4, 0, 8, 0, 0)
+    A2 = _abi.LfCsr(1 << 28, 4, 0, 8, 0, 0)
     p.block_nnz_log2[0] = 3
     assert L.lf_cell_build(ctypes.byref(A2), ctypes.byref(p), None, None, ctypes.byref(h)) == 3
     assert L.lf_spmm(None, None, 0, 4, None, 4, None) == 1
