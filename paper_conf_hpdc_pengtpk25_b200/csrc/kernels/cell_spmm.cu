@@ -37,7 +37,7 @@ constexpr unsigned kFull = 0xffffffffu;
 constexpr int kWarpsPerBlock = 8;
 constexpr int kChunk = 8;  // consecutive tasks per warp per round
 #ifndef LF_SPMM_MIN_BLOCKS
-#define LF_SPMM_MIN_BLOCKS 3
+#define LF_SPMM_MIN_BLOCKS 4
 #endif
 constexpr int kMinBlocks = LF_SPMM_MIN_BLOCKS;  // resident 256-thread blocks per SM
 
@@ -99,6 +99,10 @@ template <> struct Vec<1> {
 __device__ __forceinline__ bool tag_whole(int32_t tag) { return (tag & 7) == 7; }  // S && F && L
 __device__ __forceinline__ int32_t tag_row(int32_t tag) { return tag >> 3; }
 
+// all-zero row that padding slots (colInd = -1, val = +0.0) gather from, so
+// every slot issues the same unpredicated load (JT <= 512 floats)
+__device__ float4 g_zero_row[128];
+
 template <int VEC, int G, int NV>
 struct Layout {
     static constexpr int LPR = 32 / G;  // lanes per group
@@ -106,11 +110,12 @@ struct Layout {
     static constexpr int U = (8 / NV) > 1 ? (8 / NV) : 2;  // slots in flight per lane
 };
 
-template <int VEC, int G, int NV>
+template <int VEC, int G, int NV, bool FULL>
 struct Ctx {
     using V = Vec<VEC>;
     using VT = typename V::T;
     using L = Layout<VEC, G, NV>;
+    static constexpr int Gv = G, NVv = NV;
     const float *__restrict__ B;
     int64_t ldb;
     float *__restrict__ C;
@@ -121,11 +126,12 @@ struct Ctx {
     uint64_t pol;
 
     __device__ __forceinline__ int jcol(int m) const { return j0 + (m * L::LPR + li) * VEC; }
-    __device__ __forceinline__ bool jok(int m) const { return jcol(m) < J; }
+    __device__ __forceinline__ bool jok(int m) const { return FULL || jcol(m) < J; }
 
     __device__ __forceinline__ void gather(int32_t c, VT (&b)[NV]) const {
+        const float *r = c >= 0 ? B + (int64_t)c * ldb : reinterpret_cast<const float *>(g_zero_row) - j0;
 #pragma unroll
-        for (int m = 0; m < NV; m++) b[m] = (c >= 0 && jok(m)) ? V::load(B + (int64_t)c * ldb + jcol(m)) : V::zero();
+        for (int m = 0; m < NV; m++) b[m] = jok(m) ? V::load(r + jcol(m)) : V::zero();
     }
     // write one C row slice: plain store when this write is the row's only one
     __device__ __forceinline__ void write(int32_t row, bool plain, const VT (&acc)[NV]) const {
@@ -150,26 +156,45 @@ struct Ctx {
     }
 };
 
-// 32 slots (c_l, v_l in the lanes) accumulated into acc, no row boundary
-template <int VEC, int G, int NV>
-__device__ __forceinline__ void accum32(const Ctx<VEC, G, NV> &cx, int32_t c_l, float v_l,
-                                        typename Ctx<VEC, G, NV>::VT (&acc)[NV]) {
-    using C = Ctx<VEC, G, NV>;
-    using V = typename C::V;
-    using VT = typename C::VT;
-    constexpr int STEPS = 32 / G;
-    constexpr int U = C::L::U < STEPS ? C::L::U : STEPS;
+// Slot (col, val) pairs of the current 32-slot chunk are staged in shared
+// memory per warp, ordered so that lane group g finds its steps k, k+1
+// (slots k*G+g, (k+1)*G+g) adjacent: one broadcast LDS.128 feeds two gathers.
+template <int G>
+__device__ __forceinline__ int stage_pos(int s) { return (s % G) * (32 / G) + s / G; }
+
+template <int G>
+__device__ __forceinline__ void stage(int2 *sw, int lane, int32_t c, float v) {
+    __syncwarp();
+    sw[stage_pos<G>(lane)] = make_int2(c, __float_as_int(v));
+    __syncwarp();
+}
+
+template <class Cx, int U>
+__device__ __forceinline__ void fetch(const Cx &cx, const int2 *sw, int kb, typename Cx::VT (&b)[U][Cx::NVv],
+                                      float (&a)[U]) {
+#pragma unroll
+    for (int u = 0; u < U; u += 2) {
+        const int4 q = *reinterpret_cast<const int4 *>(sw + cx.g * (32 / Cx::Gv) + kb + u);
+        a[u] = __int_as_float(q.y);
+        cx.gather(q.x, b[u]);
+        a[u + 1] = __int_as_float(q.w);
+        cx.gather(q.z, b[u + 1]);
+    }
+}
+
+// the staged 32 slots accumulated into acc, no row boundary
+template <class Cx>
+__device__ __forceinline__ void accum32(const Cx &cx, const int2 *sw, typename Cx::VT (&acc)[Cx::NVv]) {
+    using V = typename Cx::V;
+    using VT = typename Cx::VT;
+    constexpr int NV = Cx::NVv;
+    constexpr int STEPS = 32 / Cx::Gv;
+    constexpr int U = Cx::L::U < STEPS ? Cx::L::U : STEPS;
 #pragma unroll
     for (int kb = 0; kb < STEPS; kb += U) {
         VT b[U][NV];
         float a[U];
-#pragma unroll
-        for (int u = 0; u < U; u++) {
-            const int slot = (kb + u) * G + cx.g;
-            const int32_t c = __shfl_sync(kFull, c_l, slot);
-            a[u] = __shfl_sync(kFull, v_l, slot);
-            cx.gather(c, b[u]);
-        }
+        fetch<Cx, U>(cx, sw, kb, b, a);
 #pragma unroll
         for (int u = 0; u < U; u++)
 #pragma unroll
@@ -178,30 +203,24 @@ __device__ __forceinline__ void accum32(const Ctx<VEC, G, NV> &cx, int32_t c_l, 
 }
 
 // 32-slot task of a bucket with W = 2^T < 32: 32/W CELL rows, each written.
-template <int VEC, int G, int NV, int T>
-__device__ __forceinline__ void narrow_task(const Ctx<VEC, G, NV> &cx, int32_t c_l, float v_l, int32_t tag_l) {
-    using C = Ctx<VEC, G, NV>;
-    using V = typename C::V;
-    using VT = typename C::VT;
+template <class Cx, int T>
+__device__ __forceinline__ void narrow_task(const Cx &cx, const int2 *sw, int32_t tag_l) {
+    using V = typename Cx::V;
+    using VT = typename Cx::VT;
+    constexpr int NV = Cx::NVv, G = Cx::Gv;
     constexpr int W = 1 << T;
     constexpr int STEPS = 32 / G;            // each step: one slot per group
     constexpr int RG = W >= G ? G : W;       // groups sharing one CELL row
     constexpr int SPR = W >= G ? W / G : 1;  // steps per row
-    constexpr int U = C::L::U < STEPS ? C::L::U : STEPS;
-    constexpr int LPR = C::L::LPR;
+    constexpr int U = Cx::L::U < STEPS ? Cx::L::U : STEPS;
+    constexpr int LPR = Cx::L::LPR;
     VT acc[NV];
     cx.zero(acc);
 #pragma unroll
     for (int kb = 0; kb < STEPS; kb += U) {
         VT b[U][NV];
         float a[U];
-#pragma unroll
-        for (int u = 0; u < U; u++) {
-            const int slot = (kb + u) * G + cx.g;
-            const int32_t c = __shfl_sync(kFull, c_l, slot);
-            a[u] = __shfl_sync(kFull, v_l, slot);
-            cx.gather(c, b[u]);
-        }
+        fetch<Cx, U>(cx, sw, kb, b, a);
 #pragma unroll
         for (int u = 0; u < U; u++) {
             const int step = kb + u;
@@ -224,123 +243,147 @@ __device__ __forceinline__ void narrow_task(const Ctx<VEC, G, NV> &cx, int32_t c
 struct TaskIn {
     int32_t c, tag;  // lane's slot column / row tag
     float v;
-    int b;           // bucket
+    int b;           // bucket (index into the class's table)
 };
 
-// fetch a task's slots and row tags (tasks ascend per warp, so the bucket
-// cursor only moves forward)
-__device__ __forceinline__ TaskIn load_task(const SpmmArgs &a, int64_t task, int &bcur, int lane, uint64_t pol) {
-    while (bcur + 1 < a.nb && __ldg(&a.buckets[bcur + 1].task_off) <= task) bcur++;
-    const BucketDev *bk = a.buckets + bcur;
+// W < 32 class: a task is 32 slots = 32/W rows of one bucket
+__device__ __forceinline__ TaskIn load_narrow(const SpmmArgs &a, int64_t task, int &bcur, int lane, uint64_t pol) {
+    while (bcur + 1 < a.nb_n && __ldg(&a.bk_n[bcur + 1].task_off) <= task) bcur++;
+    const BucketDev *bk = a.bk_n + bcur;
     const int64_t tin = task - __ldg(&bk->task_off);
     const int t = __ldg(&bk->t);
-    const int64_t slot_off = __ldg(&bk->slot_off), row_off = __ldg(&bk->row_off);
+    const int64_t s0 = __ldg(&bk->slot_off) + tin * 32;
+    const int64_t ns = min((int64_t)32, __ldg(&bk->n_slots) - tin * 32);
+    const int64_t nrows = ns >> t;
     TaskIn x;
     x.b = bcur;
-    if (t >= 5) {  // one CELL row of W = 2^t >= 32 slots
-        const int64_t s0 = slot_off + (tin << t);
-        x.c = ld_stream(a.col + s0 + lane, pol);
-        x.v = ld_stream(a.val + s0 + lane, pol);
-        x.tag = __shfl_sync(kFull, lane == 0 ? ld_stream(a.row_tag + row_off + tin, pol) : 0, 0);
-    } else {
-        const int64_t s0 = slot_off + tin * 32;
-        const int64_t ns = min((int64_t)32, __ldg(&bk->n_slots) - tin * 32);
-        const int64_t nrows = ns >> t;
-        x.c = lane < ns ? ld_stream(a.col + s0 + lane, pol) : -1;
-        x.v = lane < ns ? ld_stream(a.val + s0 + lane, pol) : 0.f;
-        x.tag = lane < nrows ? ld_stream(a.row_tag + row_off + ((tin * 32) >> t) + lane, pol) : -1;
-    }
+    x.c = lane < ns ? ld_stream(a.col + s0 + lane, pol) : -1;
+    x.v = lane < ns ? ld_stream(a.val + s0 + lane, pol) : 0.f;
+    x.tag = lane < nrows ? ld_stream(a.row_tag + __ldg(&bk->row_off) + ((tin * 32) >> t) + lane, pol) : -1;
     return x;
 }
 
-template <int VEC, int G, int NV>
-__global__ void __launch_bounds__(kWarpsPerBlock * 32, kMinBlocks) cell_spmm_kernel(const SpmmArgs a) {
-    using Cx = Ctx<VEC, G, NV>;
-    using VT = typename Cx::VT;
-    using L = Layout<VEC, G, NV>;
-    const int lane = threadIdx.x & 31;
-    const int64_t gwarp = (int64_t)blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
-    const int64_t nwarps = (int64_t)gridDim.x * kWarpsPerBlock;
-    const uint64_t pol = policy_evict_first();
-    Cx cx{a.B, a.ldb, a.C, a.ldc, a.J, 0, lane / L::LPR, lane % L::LPR, pol};
-    const bool single_tile = a.J <= L::JT;  // merge folded rows only without J tiling
+// W >= 32 class: a task is one CELL row; its first 32 slots are prefetched
+__device__ __forceinline__ TaskIn load_wide(const SpmmArgs &a, int64_t task, int &bcur, int lane, uint64_t pol) {
+    while (bcur + 1 < a.nb_w && __ldg(&a.bk_w[bcur + 1].task_off) <= task) bcur++;
+    const BucketDev *bk = a.bk_w + bcur;
+    const int64_t tin = task - __ldg(&bk->task_off);
+    const int64_t s0 = __ldg(&bk->slot_off) + (tin << __ldg(&bk->t));
+    TaskIn x;
+    x.b = bcur;
+    x.c = ld_stream(a.col + s0 + lane, pol);
+    x.v = ld_stream(a.val + s0 + lane, pol);
+    x.tag = lane == 0 ? ld_stream(a.row_tag + __ldg(&bk->row_off) + tin, pol) : 0;
+    return x;
+}
+
+// chunked grid-stride task order: warp w takes tasks [w*CH, w*CH+CH), then
+// advances by nwarps*CH; returns the next task and flags chunk ends
+__device__ __forceinline__ int64_t next_task(int64_t task, int64_t &cs, int64_t round, int64_t n, bool &chunk_end) {
+    int64_t tn = task + 1;
+    chunk_end = false;
+    if (tn >= cs + kChunk || tn >= n) {
+        chunk_end = true;
+        cs += round;
+        tn = cs;
+    }
+    return tn;
+}
+
+template <class Cx>
+__device__ __forceinline__ void narrow_loop(const SpmmArgs &a, const Cx &cx0, int2 *sw, int lane, int64_t wid,
+                                            int64_t nw, uint64_t pol) {
+    Cx cx = cx0;
+    constexpr int JT = Cx::L::JT;
+    const int64_t round = nw * kChunk;
+    int64_t cs = wid * kChunk;
+    if (cs >= a.n_tasks_n) return;
     int bcur = 0;
-
-    VT acc[NV];
-    cx.zero(acc);
-    int32_t pend = -1;  // tag of the run being accumulated in acc (-1: none)
-    bool run_first = false;
-
-    const int64_t round = nwarps * kChunk;
-    int64_t cs = gwarp * kChunk;  // chunk start
-    if (cs >= a.n_tasks) return;
     int64_t task = cs;
-    TaskIn cur = load_task(a, task, bcur, lane, pol);
-    while (task < a.n_tasks) {
-        int64_t tn = task + 1;
-        bool chunk_end = false;
-        if (tn >= cs + kChunk || tn >= a.n_tasks) {
-            chunk_end = true;
-            cs += round;
-            tn = cs;
-        }
+    TaskIn cur = load_narrow(a, task, bcur, lane, pol);
+    while (task < a.n_tasks_n) {
+        bool chunk_end;
+        const int64_t tn = next_task(task, cs, round, a.n_tasks_n, chunk_end);
         TaskIn nxt{};
-        if (tn < a.n_tasks) nxt = load_task(a, tn, bcur, lane, pol);
-        const int t = __ldg(&a.buckets[cur.b].t);
-        if (t >= 5) {
-            const int32_t tag = cur.tag;
-            if (tag >= 0) {
-                if (pend >= 0 && tag_row(pend) != tag_row(tag)) {
-                    cx.reduce_groups(acc);
-                    if (cx.g == 0) cx.write(tag_row(pend), false, acc);
-                    cx.zero(acc);
-                    pend = -1;
-                }
-                if (pend < 0) run_first = (tag & 2) != 0;
-                const int64_t W = int64_t(1) << t;
-                const int64_t s0 = __ldg(&a.buckets[cur.b].slot_off) + ((task - __ldg(&a.buckets[cur.b].task_off)) << t);
-                for (int j0 = 0; j0 < a.J; j0 += L::JT) {
-                    cx.j0 = j0;
-                    if (!single_tile) cx.zero(acc);
-                    accum32<VEC, G, NV>(cx, cur.c, cur.v, acc);
-                    for (int64_t base = 32; base < W; base += 32) {
-                        const int32_t c_l = ld_stream(a.col + s0 + base + lane, pol);
-                        const float v_l = ld_stream(a.val + s0 + base + lane, pol);
-                        if (__ballot_sync(kFull, c_l >= 0) == 0) break;  // rest is padding
-                        accum32<VEC, G, NV>(cx, c_l, v_l, acc);
-                    }
-                    if (!single_tile) {  // no run merging across J tiles
-                        cx.reduce_groups(acc);
-                        if (cx.g == 0) cx.write(tag_row(tag), tag_whole(tag), acc);
-                    }
-                }
-                if (single_tile) {
-                    pend = tag;
-                    if (tag & 1) {  // last sub-row of the segment completes the run
-                        cx.reduce_groups(acc);
-                        if (cx.g == 0) cx.write(tag_row(tag), run_first && (tag & 4), acc);
-                        cx.zero(acc);
-                        pend = -1;
-                    }
+        if (tn < a.n_tasks_n) nxt = load_narrow(a, tn, bcur, lane, pol);
+        if (__ballot_sync(kFull, cur.tag >= 0)) {
+            const int t = __ldg(&a.bk_n[cur.b].t);
+            stage<Cx::Gv>(sw, lane, cur.c, cur.v);
+            for (int j0 = 0; j0 < a.J; j0 += JT) {
+                cx.j0 = j0;
+                switch (t) {
+                case 0: narrow_task<Cx, 0>(cx, sw, cur.tag); break;
+                case 1: narrow_task<Cx, 1>(cx, sw, cur.tag); break;
+                case 2: narrow_task<Cx, 2>(cx, sw, cur.tag); break;
+                case 3: narrow_task<Cx, 3>(cx, sw, cur.tag); break;
+                default: narrow_task<Cx, 4>(cx, sw, cur.tag); break;
                 }
             }
-        } else {
-            if (pend >= 0) {
+        }
+        task = tn;
+        cur = nxt;
+    }
+}
+
+template <class Cx>
+__device__ __forceinline__ void wide_loop(const SpmmArgs &a, const Cx &cx0, int2 *sw, int lane, int64_t wid,
+                                          int64_t nw, uint64_t pol) {
+    using VT = typename Cx::VT;
+    constexpr int NV = Cx::NVv, G = Cx::Gv, JT = Cx::L::JT;
+    Cx cx = cx0;
+    const bool single_tile = a.J <= JT;  // merge folded rows only without J tiling
+    const int64_t round = nw * kChunk;
+    int64_t cs = wid * kChunk;
+    if (cs >= a.n_tasks_w) return;
+    int bcur = 0;
+    int64_t task = cs;
+    TaskIn cur = load_wide(a, task, bcur, lane, pol);
+    VT acc[NV];
+    cx.zero(acc);
+    int32_t pend = -1;  // tag of the run accumulated in acc (-1: none)
+    bool run_first = false;
+    while (task < a.n_tasks_w) {
+        bool chunk_end;
+        const int64_t tn = next_task(task, cs, round, a.n_tasks_w, chunk_end);
+        TaskIn nxt{};
+        if (tn < a.n_tasks_w) nxt = load_wide(a, tn, bcur, lane, pol);
+        const int32_t tag = __shfl_sync(kFull, cur.tag, 0);
+        if (tag >= 0) {
+            if (pend >= 0 && tag_row(pend) != tag_row(tag)) {  // previous run split off: red
                 cx.reduce_groups(acc);
                 if (cx.g == 0) cx.write(tag_row(pend), false, acc);
                 cx.zero(acc);
                 pend = -1;
             }
-            if (__ballot_sync(kFull, cur.tag >= 0)) {
-                for (int j0 = 0; j0 < a.J; j0 += L::JT) {
-                    cx.j0 = j0;
-                    switch (t) {
-                    case 0: narrow_task<VEC, G, NV, 0>(cx, cur.c, cur.v, cur.tag); break;
-                    case 1: narrow_task<VEC, G, NV, 1>(cx, cur.c, cur.v, cur.tag); break;
-                    case 2: narrow_task<VEC, G, NV, 2>(cx, cur.c, cur.v, cur.tag); break;
-                    case 3: narrow_task<VEC, G, NV, 3>(cx, cur.c, cur.v, cur.tag); break;
-                    default: narrow_task<VEC, G, NV, 4>(cx, cur.c, cur.v, cur.tag); break;
-                    }
+            if (pend < 0) run_first = (tag & 2) != 0;
+            const BucketDev *bk = a.bk_w + cur.b;
+            const int t = __ldg(&bk->t);
+            const int64_t s0 = __ldg(&bk->slot_off) + ((task - __ldg(&bk->task_off)) << t);
+            const int64_t W = int64_t(1) << t;
+            for (int j0 = 0; j0 < a.J; j0 += JT) {
+                cx.j0 = j0;
+                stage<G>(sw, lane, cur.c, cur.v);
+                accum32(cx, sw, acc);
+                for (int64_t base = 32; base < W; base += 32) {
+                    const int32_t c_l = ld_stream(a.col + s0 + base + lane, pol);
+                    const float v_l = ld_stream(a.val + s0 + base + lane, pol);
+                    if (__ballot_sync(kFull, c_l >= 0) == 0) break;  // rest is padding
+                    stage<G>(sw, lane, c_l, v_l);
+                    accum32(cx, sw, acc);
+                }
+                if (!single_tile) {  // J tiles: every tile writes its own slice
+                    cx.reduce_groups(acc);
+                    if (cx.g == 0) cx.write(tag_row(tag), tag_whole(tag), acc);
+                    cx.zero(acc);
+                }
+            }
+            if (single_tile) {
+                pend = tag;
+                if (tag & 1) {  // last sub-row of the segment completes the run
+                    cx.reduce_groups(acc);
+                    if (cx.g == 0) cx.write(tag_row(tag), run_first && (tag & 4), acc);
+                    cx.zero(acc);
+                    pend = -1;
                 }
             }
         }
@@ -355,16 +398,38 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kMinBlocks) cell_spmm_ker
     }
 }
 
+// Blocks [0, a.blocks_n) run the W < 32 tasks, the rest the W >= 32 tasks:
+// the two loops share no live state, so each is register-allocated alone.
+template <int VEC, int G, int NV, bool FULL>
+__global__ void __launch_bounds__(kWarpsPerBlock * 32, kMinBlocks) cell_spmm_kernel(const SpmmArgs a) {
+    using Cx = Ctx<VEC, G, NV, FULL>;
+    using L = Layout<VEC, G, NV>;
+    __shared__ __align__(16) int2 stage_buf[kWarpsPerBlock][32];
+    const int lane = threadIdx.x & 31;
+    int2 *sw = stage_buf[threadIdx.x >> 5];
+    const uint64_t pol = policy_evict_first();
+    const Cx cx{a.B, a.ldb, a.C, a.ldc, a.J, 0, lane / L::LPR, lane % L::LPR, pol};
+    const int w = threadIdx.x >> 5;
+    if ((int)blockIdx.x < a.blocks_n)
+        narrow_loop(a, cx, sw, lane, (int64_t)blockIdx.x * kWarpsPerBlock + w, (int64_t)a.blocks_n * kWarpsPerBlock,
+                    pol);
+    else
+        wide_loop(a, cx, sw, lane, (int64_t)(blockIdx.x - a.blocks_n) * kWarpsPerBlock + w,
+                  (int64_t)(gridDim.x - a.blocks_n) * kWarpsPerBlock, pol);
+}
+
 // Algorithm 1 on the GPU straight from CSR: one warp per row, same lane layout.
-template <int VEC, int G, int NV>
+template <int VEC, int G, int NV, bool FULL>
 __global__ void __launch_bounds__(kWarpsPerBlock * 32)
     csr_spmm_kernel(const int64_t *__restrict__ row_ptr, const int32_t *__restrict__ col,
                     const float *__restrict__ val, int64_t n_rows, const float *__restrict__ B, int64_t ldb,
                     float *__restrict__ C, int64_t ldc, int J) {
-    using Cx = Ctx<VEC, G, NV>;
+    using Cx = Ctx<VEC, G, NV, FULL>;
     using VT = typename Cx::VT;
     using L = Layout<VEC, G, NV>;
+    __shared__ __align__(16) int2 stage_buf[kWarpsPerBlock][32];
     const int lane = threadIdx.x & 31;
+    int2 *sw = stage_buf[threadIdx.x >> 5];
     const int64_t gwarp = (int64_t)blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
     const int64_t nwarps = (int64_t)gridDim.x * kWarpsPerBlock;
     const uint64_t pol = policy_evict_first();
@@ -377,9 +442,9 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32)
             cx.zero(acc);
             for (int64_t base = rb; base < re; base += 32) {
                 const bool in = base + lane < re;
-                const int32_t c_l = in ? ld_stream(col + base + lane, pol) : -1;
-                const float v_l = in ? ld_stream(val + base + lane, pol) : 0.f;
-                accum32<VEC, G, NV>(cx, c_l, v_l, acc);
+                stage<G>(sw, lane, in ? ld_stream(col + base + lane, pol) : -1,
+                         in ? ld_stream(val + base + lane, pol) : 0.f);
+                accum32(cx, sw, acc);
             }
             cx.reduce_groups(acc);
             if (cx.g == 0) cx.write((int32_t)i, true, acc);
@@ -420,26 +485,48 @@ int resident_blocks(F fn) {
     return std::max(1, occ) * std::max(1, sms);
 }
 
-template <int VEC, int G, int NV>
-cudaError_t run_cell(const SpmmArgs &a, cudaStream_t s) {
+template <int VEC, int G, int NV, bool FULL>
+cudaError_t run_cell(const SpmmArgs &a0, cudaStream_t s) {
     static int cap = 0;
-    auto fn = cell_spmm_kernel<VEC, G, NV>;
+    auto fn = cell_spmm_kernel<VEC, G, NV, FULL>;
     if (!cap) cap = resident_blocks(fn);
-    int64_t want = (a.n_tasks + kWarpsPerBlock * kChunk - 1) / (kWarpsPerBlock * kChunk);
-    int grid = (int)std::max<int64_t>(1, std::min<int64_t>(want, cap));
+    SpmmArgs a = a0;
+    const int64_t per_block = kWarpsPerBlock * kChunk;
+    const int64_t want_n = (a.n_tasks_n + per_block - 1) / per_block;
+    const int64_t want_w = (a.n_tasks_w + per_block - 1) / per_block;
+    // split the resident blocks in proportion to the slots of each class
+    const double frac_n = a.slots_n + a.slots_w > 0 ? (double)a.slots_n / (double)(a.slots_n + a.slots_w) : 0.0;
+    int64_t bn = want_n ? std::max<int64_t>(1, (int64_t)(frac_n * cap + 0.5)) : 0;
+    int64_t bw = want_w ? std::max<int64_t>(1, cap - bn) : 0;
+    bn = std::min(bn, want_n);
+    bw = std::min(bw, want_w);
+    a.blocks_n = (int)bn;
+    const int grid = (int)(bn + bw);
+    if (grid == 0) return cudaSuccess;
     fn<<<grid, kWarpsPerBlock * 32, 0, s>>>(a);
     return cudaGetLastError();
 }
 
 template <int VEC, int G, int NV>
+cudaError_t run_cell_j(const SpmmArgs &a, cudaStream_t s) {
+    return a.J == Layout<VEC, G, NV>::JT ? run_cell<VEC, G, NV, true>(a, s) : run_cell<VEC, G, NV, false>(a, s);
+}
+
+template <int VEC, int G, int NV, bool FULL>
 cudaError_t run_csr(const lf_csr &A, const float *B, int64_t ldb, int J, float *C, int64_t ldc, cudaStream_t s) {
     static int cap = 0;
-    auto fn = csr_spmm_kernel<VEC, G, NV>;
+    auto fn = csr_spmm_kernel<VEC, G, NV, FULL>;
     if (!cap) cap = resident_blocks(fn);
     int64_t want = (A.n_rows + kWarpsPerBlock - 1) / kWarpsPerBlock;
     int grid = (int)std::max<int64_t>(1, std::min<int64_t>(want, cap));
     fn<<<grid, kWarpsPerBlock * 32, 0, s>>>(A.row_ptr, A.col_ind, A.val, A.n_rows, B, ldb, C, ldc, J);
     return cudaGetLastError();
+}
+
+template <int VEC, int G, int NV>
+cudaError_t run_csr_j(const lf_csr &A, const float *B, int64_t ldb, int J, float *C, int64_t ldc, cudaStream_t s) {
+    return J == Layout<VEC, G, NV>::JT ? run_csr<VEC, G, NV, true>(A, B, ldb, J, C, ldc, s)
+                                       : run_csr<VEC, G, NV, false>(A, B, ldb, J, C, ldc, s);
 }
 
 bool vec4_ok(const float *B, int64_t ldb, const float *C, int64_t ldc, int J) {
@@ -458,28 +545,28 @@ cudaError_t launch_zero_rows(const int32_t *row_cnt, int64_t n_rows, float *C, i
 }
 
 cudaError_t launch_cell_spmm(const SpmmArgs &a, cudaStream_t s) {
-    if (a.n_tasks == 0 || a.J == 0) return cudaSuccess;
+    if (a.n_tasks_n + a.n_tasks_w == 0 || a.J == 0) return cudaSuccess;
     if (vec4_ok(a.B, a.ldb, a.C, a.ldc, a.J)) {
-        if (a.J <= 32) return run_cell<4, 4, 1>(a, s);
-        if (a.J <= 64) return run_cell<4, 2, 1>(a, s);
-        if (a.J <= 128) return run_cell<4, 1, 1>(a, s);
-        if (a.J <= 256) return run_cell<4, 1, 2>(a, s);
-        return run_cell<4, 1, 4>(a, s);
+        if (a.J <= 32) return run_cell_j<4, 4, 1>(a, s);
+        if (a.J <= 64) return run_cell_j<4, 2, 1>(a, s);
+        if (a.J <= 128) return run_cell_j<4, 1, 1>(a, s);
+        if (a.J <= 256) return run_cell_j<4, 1, 2>(a, s);
+        return run_cell_j<4, 1, 4>(a, s);
     }
-    return run_cell<1, 1, 4>(a, s);
+    return run_cell<1, 1, 4, false>(a, s);
 }
 
 cudaError_t launch_csr_spmm(const lf_csr &A, const float *B, int64_t ldb, int J, float *C, int64_t ldc,
                             cudaStream_t s) {
     if (A.n_rows == 0 || J == 0) return cudaSuccess;
     if (vec4_ok(B, ldb, C, ldc, J)) {
-        if (J <= 32) return run_csr<4, 4, 1>(A, B, ldb, J, C, ldc, s);
-        if (J <= 64) return run_csr<4, 2, 1>(A, B, ldb, J, C, ldc, s);
-        if (J <= 128) return run_csr<4, 1, 1>(A, B, ldb, J, C, ldc, s);
-        if (J <= 256) return run_csr<4, 1, 2>(A, B, ldb, J, C, ldc, s);
-        return run_csr<4, 1, 4>(A, B, ldb, J, C, ldc, s);
+        if (J <= 32) return run_csr_j<4, 4, 1>(A, B, ldb, J, C, ldc, s);
+        if (J <= 64) return run_csr_j<4, 2, 1>(A, B, ldb, J, C, ldc, s);
+        if (J <= 128) return run_csr_j<4, 1, 1>(A, B, ldb, J, C, ldc, s);
+        if (J <= 256) return run_csr_j<4, 1, 2>(A, B, ldb, J, C, ldc, s);
+        return run_csr_j<4, 1, 4>(A, B, ldb, J, C, ldc, s);
     }
-    return run_csr<1, 1, 4>(A, B, ldb, J, C, ldc, s);
+    return run_csr<1, 1, 4, false>(A, B, ldb, J, C, ldc, s);
 }
 
 }  // namespace lf

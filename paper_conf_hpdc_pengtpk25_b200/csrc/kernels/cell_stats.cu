@@ -106,47 +106,61 @@ __global__ void __launch_bounds__(kThreads) stats_rows_kernel(const int64_t *__r
     }
 }
 
-// nnz-balanced column marking.  Positions q of tile [q0, q0 + kMarkTile) are
-// mapped to their row by a binary search in row_ptr restricted to the tile's
-// row range (found once per block).
+// nnz-balanced column marking.  Every lane owns kMarkPerThread consecutive
+// positions: one binary search in row_ptr finds the row of its first
+// position, then rows advance as positions cross row_ptr boundaries.
+// Power-law inputs send a large share of all nonzeros to a few hot columns
+// whose mask words share L2 lines, so a per-block direct-mapped filter in
+// shared memory ((col << 32) | bits already set globally, one 64-bit word per
+// slot, updated with whole-word stores so a (col, bits) pair is always
+// consistent) drops repeated (col, bit) pairs before they reach L2.
+constexpr int kFilter = 4096;
+
 __global__ void __launch_bounds__(kThreads) stats_mark_kernel(const int64_t *__restrict__ row_ptr,
                                                               const int32_t *__restrict__ col, int64_t n_rows,
                                                               int64_t S, int P,
                                                               const uint8_t *__restrict__ t0seg,
                                                               uint32_t *__restrict__ mask) {
-    __shared__ int64_t rng[2];
+    __shared__ unsigned long long filt[kFilter];
+    for (int q = threadIdx.x; q < kFilter; q += blockDim.x) filt[q] = ~0ull;  // col field 0xFFFFFFFF: empty
+    __syncthreads();
     const int64_t base = row_ptr[0];
     const int64_t nnz = row_ptr[n_rows] - base;
-    for (int64_t q0 = (int64_t)blockIdx.x * kMarkTile; q0 < nnz; q0 += (int64_t)gridDim.x * kMarkTile) {
-        if (threadIdx.x < 2) {
-            // last row r with row_ptr[r] - base <= target
-            const int64_t target = threadIdx.x == 0 ? q0 : min(q0 + kMarkTile, nnz) - 1;
-            int64_t lo = 0, hi = n_rows - 1;
-            while (lo < hi) {
-                int64_t m = (lo + hi + 1) >> 1;
-                if (row_ptr[m] - base <= target) lo = m;
-                else hi = m - 1;
-            }
-            rng[threadIdx.x] = lo;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x * kMarkPerThread;
+    for (int64_t q0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * kMarkPerThread; q0 < nnz; q0 += stride) {
+        // row of position q0: last r with row_ptr[r] - base <= q0
+        int64_t lo = 0, hi = n_rows - 1;
+        while (lo < hi) {
+            const int64_t m = (lo + hi + 1) >> 1;
+            if (__ldg(row_ptr + m) - base <= q0) lo = m;
+            else hi = m - 1;
         }
-        __syncthreads();
-        const int64_t rlo = rng[0], rhi = rng[1];
-#pragma unroll 4
+        int64_t r = lo;
+        int64_t rend = __ldg(row_ptr + r + 1) - base;
+        int32_t c[kMarkPerThread];
+        uint32_t bit[kMarkPerThread];
+#pragma unroll
         for (int k = 0; k < kMarkPerThread; k++) {
-            const int64_t q = q0 + k * kThreads + threadIdx.x;
-            if (q >= nnz) break;
-            int64_t lo = rlo, hi = rhi;
-            while (lo < hi) {
-                int64_t m = (lo + hi + 1) >> 1;
-                if (row_ptr[m] - base <= q) lo = m;
-                else hi = m - 1;
+            const int64_t q = q0 + k;
+            c[k] = -1;
+            bit[k] = 0;
+            if (q < nnz) {
+                while (q >= rend) rend = __ldg(row_ptr + (++r) + 1) - base;
+                c[k] = __ldg(col + base + q);
+                const int p = P == 1 ? 0 : (int)(c[k] / S);
+                bit[k] = 1u << __ldg(t0seg + r * P + p);
             }
-            const int32_t c = col[base + q];
-            const int p = P == 1 ? 0 : (int)(c / S);
-            const uint32_t bit = 1u << t0seg[lo * P + p];
-            if (!(__ldcg(mask + c) & bit)) atomicOr(mask + c, bit);
         }
-        __syncthreads();
+#pragma unroll
+        for (int k = 0; k < kMarkPerThread; k++) {
+            if (c[k] < 0) continue;
+            const int slot = c[k] & (kFilter - 1);
+            const unsigned long long f = filt[slot];
+            const bool same = (uint32_t)(f >> 32) == (uint32_t)c[k];
+            if (same && ((uint32_t)f & bit[k])) continue;
+            atomicOr(mask + c[k], bit[k]);
+            filt[slot] = ((unsigned long long)(uint32_t)c[k] << 32) | (same ? ((uint32_t)f | bit[k]) : bit[k]);
+        }
     }
 }
 
@@ -210,7 +224,7 @@ cudaError_t launch_stats(const lf_csr &A, int P, StatsDev *d_stats, uint32_t *d_
         stats_rows_kernel<<<grid, kThreads, smem, s>>>(A.row_ptr, A.col_ind, A.n_rows, S, P, d_stats, d_t0seg);
         if (A.nnz > 0) {
             int64_t tiles = (A.nnz + kMarkTile - 1) / kMarkTile;
-            int g2 = (int)std::min<int64_t>(tiles, (int64_t)num_sms() * 8);
+            int g2 = (int)std::min<int64_t>(tiles, (int64_t)num_sms() * 16);
             stats_mark_kernel<<<g2, kThreads, 0, s>>>(A.row_ptr, A.col_ind, A.n_rows, S, P, d_t0seg, d_colmask);
         }
     }

@@ -60,6 +60,22 @@ struct Scratch {
     }
 };
 
+// The device's default stream-ordered pool (cudaMallocAsync, used for the
+// configure scratch and when no lf_allocator is given) returns memory to the
+// OS at every synchronisation unless its release threshold is raised; a
+// re-map costs milliseconds, so keep the pool's memory (once per device).
+void keep_default_pool() {
+    static bool done[64] = {};
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64 || done[dev]) return;
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+        uint64_t thr = UINT64_MAX;
+        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+    }
+    done[dev] = true;
+}
+
 lf_status check_csr(const lf_csr *A) {
     if (!A) return fail(LF_ERR_INVALID_ARG, "A is NULL");
     if (A->n_rows < 0 || A->n_cols < 0 || A->nnz < 0) return fail(LF_ERR_INVALID_ARG, "negative size");
@@ -144,6 +160,7 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
     cudaStream_t s = (cudaStream_t)stream;
     if (lf_status st = maybe_validate(A, s)) return st;
 
+    keep_default_pool();
     const int P = o.force_parts ? o.force_parts : standin_parts(A, J, max_parts);
     lf::StatsDev *d_st = nullptr;
     uint32_t *d_mask = nullptr;
@@ -233,6 +250,7 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
     if (al && (!al->alloc || !al->free)) return fail(LF_ERR_INVALID_ARG, "allocator without alloc/free");
     cudaStream_t s = (cudaStream_t)stream;
     if (lf_status st = maybe_validate(A, s)) return st;
+    keep_default_pool();
 
     lf_cell *h = new lf_cell();
     h->params = *params;
@@ -291,7 +309,8 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
 
     // host: bucket table (R2, R7) and warp-task decomposition
     std::vector<long long> row_off((size_t)P * lf::kMaxT, -1);
-    int64_t R_tot = 0, S_tot = 0, tasks = 0;
+    int64_t R_tot = 0, S_tot = 0;
+    std::vector<lf::BucketDev> bn, bw;
     for (int p = 0; p < P; p++) {
         const int k = params->block_nnz_log2[p];
         for (int t = 0; t <= params->max_width_log2[p]; t++) {
@@ -312,19 +331,32 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
             d.slot_off = S_tot;
             d.row_off = R_tot;
             d.n_slots = pad * W;
-            d.task_off = tasks;
             d.t = t;
             d.task_slots = (int32_t)std::max<int64_t>(32, W);
+            if (W < 32) {
+                d.task_off = h->n_tasks_n;
+                h->n_tasks_n += (pad * W + 31) / 32;
+                h->slots_n += pad * W;
+                bn.push_back(d);
+            } else {
+                d.task_off = h->n_tasks_w;
+                h->n_tasks_w += pad;
+                h->slots_w += pad * W;
+                bw.push_back(d);
+            }
+            d.task_off = 0;
             h->h_buckets.push_back(d);
             row_off[(size_t)p * lf::kMaxT + t] = R_tot;
-            tasks += W <= 32 ? (pad * W + 31) / 32 : pad;
             R_tot += pad;
             S_tot += pad * W;
         }
     }
     h->n_cell_rows = R_tot;
     h->n_slots = S_tot;
-    h->n_tasks = tasks;
+    h->nb_n = (int)bn.size();
+    h->nb_w = (int)bw.size();
+    h->h_buckets.insert(h->h_buckets.end(), bn.begin(), bn.end());
+    h->h_buckets.insert(h->h_buckets.end(), bw.begin(), bw.end());
     const int nb = (int)h->buckets.size();
     if (nb > 2048) return bail(fail(LF_ERR_UNSUPPORTED, "more than 2048 buckets"));
 
@@ -332,7 +364,7 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
     const size_t a256 = 256;
     auto up = [&](size_t b) { return (b + a256 - 1) / a256 * a256; };
     const size_t b_ri = up(R_tot * 4), b_rt = up(R_tot * 4), b_ci = up(S_tot * 4), b_va = up(S_tot * 4),
-                 b_bk = up(nb * sizeof(lf::BucketDev));
+                 b_bk = up(h->h_buckets.size() * sizeof(lf::BucketDev));
     h->pool_bytes = b_ri + b_rt + b_ci + b_va + b_bk;
     h->pool = mem.get(h->pool_bytes);
     if (h->pool_bytes && !h->pool) return bail(fail(LF_ERR_NO_MEMORY, "CELL arrays allocation failed"));
@@ -351,7 +383,7 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
         if ((st = cu(cudaMemsetAsync(h->row_tag, 0xFF, R_tot * 4, s), "memset"))) return bail(st);
         if ((st = cu(cudaMemsetAsync(bs.src_cnt, 0, R_tot * 4, s), "memset"))) return bail(st);
     }
-    if (nb && (st = cu(cudaMemcpyAsync(h->d_buckets, h->h_buckets.data(), nb * sizeof(lf::BucketDev),
+    if (nb && (st = cu(cudaMemcpyAsync(h->d_buckets, h->h_buckets.data(), h->h_buckets.size() * sizeof(lf::BucketDev),
                                        cudaMemcpyHostToDevice, s),
                        "H2D buckets")))
         return bail(st);
@@ -381,8 +413,9 @@ lf_status lf_spmm(const lf_cell *h, const float *B, int64_t ldb, int32_t J, floa
         return LF_OK;
     }
     LF_CUDA(lf::launch_zero_rows(h->row_cnt, h->n_rows, C, ldc, J, s));
-    lf::SpmmArgs a{h->d_buckets, (int)h->buckets.size(), h->n_tasks, h->col_ind, h->val, h->row_tag,
-                   B, ldb, C, ldc, J};
+    const int nb = (int)h->buckets.size();
+    lf::SpmmArgs a{h->d_buckets + nb, h->d_buckets + nb + h->nb_n, h->nb_n, h->nb_w, h->n_tasks_n, h->n_tasks_w,
+                   h->slots_n, h->slots_w, 0, h->col_ind, h->val, h->row_tag, B, ldb, C, ldc, J};
     LF_CUDA(lf::launch_cell_spmm(a, s));
     return LF_OK;
 }

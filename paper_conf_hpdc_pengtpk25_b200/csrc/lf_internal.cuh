@@ -71,9 +71,12 @@ cudaError_t launch_slot_fill(const lf_csr &A, const BucketDev *d_buckets, int nb
 
 // SpMM
 struct SpmmArgs {
-    const BucketDev *buckets;
-    int nb;
-    int64_t n_tasks;
+    const BucketDev *bk_n;  // buckets with W < 32; task_off counts 32-slot tasks
+    const BucketDev *bk_w;  // buckets with W >= 32; task_off counts rows
+    int nb_n, nb_w;
+    int64_t n_tasks_n, n_tasks_w;
+    int64_t slots_n, slots_w;
+    int blocks_n;  // set by the launcher
     const int32_t *col;
     const float *val;
     const int32_t *row_tag;
@@ -94,13 +97,15 @@ cudaError_t launch_validate(const lf_csr &A, int *d_flag, cudaStream_t s);
 struct lf_cell {
     lf_cell_params params;
     int64_t n_rows = 0, n_cols = 0, nnz = 0;
-    int64_t n_cell_rows = 0, n_slots = 0, n_tasks = 0;
+    int64_t n_cell_rows = 0, n_slots = 0;
+    int64_t n_tasks_n = 0, n_tasks_w = 0, slots_n = 0, slots_w = 0;
+    int nb_n = 0, nb_w = 0;
     int32_t *row_ind = nullptr;  // view array (bit-exact with the oracle)
     int32_t *col_ind = nullptr;
     float *val = nullptr;
     int32_t *row_tag = nullptr;  // (row << 3) | S,F,L flags (cell_spmm.cu); -1 = padding
     int32_t *row_cnt = nullptr;  // CELL rows per source row
-    lf::BucketDev *d_buckets = nullptr;
+    lf::BucketDev *d_buckets = nullptr;  // [nb] all, then [nb_n] W < 32 class, then [nb_w] W >= 32 class
     std::vector<lf_bucket> buckets;
     std::vector<lf::BucketDev> h_buckets;
     // memory: one pool allocation holds every array above
