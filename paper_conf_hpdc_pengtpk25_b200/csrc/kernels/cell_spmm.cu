@@ -128,8 +128,12 @@ struct Ctx {
     __device__ __forceinline__ int jcol(int m) const { return j0 + (m * L::LPR + li) * VEC; }
     __device__ __forceinline__ bool jok(int m) const { return FULL || jcol(m) < J; }
 
-    __device__ __forceinline__ void gather(int32_t c, VT (&b)[NV]) const {
-        const float *r = c >= 0 ? B + (int64_t)c * ldb : reinterpret_cast<const float *>(g_zero_row) - j0;
+    // address of B row c, or of the zero row for a padding slot (computed once
+    // per slot when a chunk is resolved, not in the gather loop)
+    __device__ __forceinline__ const float *rowaddr(int32_t c) const {
+        return c >= 0 ? B + (int64_t)c * ldb : reinterpret_cast<const float *>(g_zero_row) - j0;
+    }
+    __device__ __forceinline__ void gather(const float *r, VT (&b)[NV]) const {
 #pragma unroll
         for (int m = 0; m < NV; m++) b[m] = jok(m) ? V::load(r + jcol(m)) : V::zero();
     }
@@ -156,35 +160,55 @@ struct Ctx {
     }
 };
 
-// Slot (col, val) pairs of the current 32-slot chunk are staged in shared
-// memory per warp, ordered so that lane group g finds its steps k, k+1
-// (slots k*G+g, (k+1)*G+g) adjacent: one broadcast LDS.128 feeds two gathers.
+// The current 32-slot chunk is RESOLVED in shared memory per warp: every
+// slot's B-row address (zero row for padding) and value, ordered so that lane
+// group g finds its steps k, k+1 (slots k*G+g, (k+1)*G+g) adjacent -- one
+// broadcast LDS.128 + one LDS.64 feed two gathers.
+struct Resolved {
+    const float *addr[32];
+    float val[32];
+};
+
 template <int G>
 __device__ __forceinline__ int stage_pos(int s) { return (s % G) * (32 / G) + s / G; }
 
-template <int G>
-__device__ __forceinline__ void stage(int2 *sw, int lane, int32_t c, float v) {
+// synchronous path: (c, v) of the lane's slot from registers
+template <int G, class Cx>
+__device__ __forceinline__ void stage(const Cx &cx, Resolved &r, int lane, int32_t c, float v) {
     __syncwarp();
-    sw[stage_pos<G>(lane)] = make_int2(c, __float_as_int(v));
+    const int p = stage_pos<G>(lane);
+    r.addr[p] = cx.rowaddr(c);
+    r.val[p] = v;
+    __syncwarp();
+}
+
+// asynchronous path: raw (c, v bits) already landed at stage positions
+template <class Cx>
+__device__ __forceinline__ void resolve(const Cx &cx, const int2 *raw, Resolved &r, int lane) {
+    const int2 e = raw[lane];
+    r.addr[lane] = cx.rowaddr(e.x);
+    r.val[lane] = __int_as_float(e.y);
     __syncwarp();
 }
 
 template <class Cx, int U>
-__device__ __forceinline__ void fetch(const Cx &cx, const int2 *sw, int kb, typename Cx::VT (&b)[U][Cx::NVv],
+__device__ __forceinline__ void fetch(const Cx &cx, const Resolved &r, int kb, typename Cx::VT (&b)[U][Cx::NVv],
                                       float (&a)[U]) {
 #pragma unroll
     for (int u = 0; u < U; u += 2) {
-        const int4 q = *reinterpret_cast<const int4 *>(sw + cx.g * (32 / Cx::Gv) + kb + u);
-        a[u] = __int_as_float(q.y);
-        cx.gather(q.x, b[u]);
-        a[u + 1] = __int_as_float(q.w);
-        cx.gather(q.z, b[u + 1]);
+        const int p = cx.g * (32 / Cx::Gv) + kb + u;
+        const ulonglong2 ad = *reinterpret_cast<const ulonglong2 *>(&r.addr[p]);
+        const float2 vv = *reinterpret_cast<const float2 *>(&r.val[p]);
+        a[u] = vv.x;
+        cx.gather(reinterpret_cast<const float *>(ad.x), b[u]);
+        a[u + 1] = vv.y;
+        cx.gather(reinterpret_cast<const float *>(ad.y), b[u + 1]);
     }
 }
 
 // the staged 32 slots accumulated into acc, no row boundary
 template <class Cx>
-__device__ __forceinline__ void accum32(const Cx &cx, const int2 *sw, typename Cx::VT (&acc)[Cx::NVv]) {
+__device__ __forceinline__ void accum32(const Cx &cx, const Resolved &sw, typename Cx::VT (&acc)[Cx::NVv]) {
     using V = typename Cx::V;
     using VT = typename Cx::VT;
     constexpr int NV = Cx::NVv;
@@ -204,7 +228,7 @@ __device__ __forceinline__ void accum32(const Cx &cx, const int2 *sw, typename C
 
 // 32-slot task of a bucket with W = 2^T < 32: 32/W CELL rows, each written.
 template <class Cx, int T>
-__device__ __forceinline__ void narrow_task(const Cx &cx, const int2 *sw, int32_t tag_l) {
+__device__ __forceinline__ void narrow_task(const Cx &cx, const Resolved &sw, int32_t tag_l) {
     using V = typename Cx::V;
     using VT = typename Cx::VT;
     constexpr int NV = Cx::NVv, G = Cx::Gv;
@@ -240,45 +264,28 @@ __device__ __forceinline__ void narrow_task(const Cx &cx, const int2 *sw, int32_
     }
 }
 
-struct TaskIn {
-    int32_t c, tag;  // lane's slot column / row tag
-    float v;
-    int b;           // bucket (index into the class's table)
+// ---- asynchronous staging ----------------------------------------------
+// A warp owns two stage buffers; while it gathers B rows for the slots in
+// one, cp.async (LDGSTS, L2 evict_first) fills the other with the next
+// 32 slots (and their row tags), so the index/value stream never waits in
+// registers.
+struct WarpStage {
+    int2 slot[2][32];   // raw (col, val bits) at stage_pos order, filled by cp.async
+    int32_t tag[2][32]; // row tags of the staged slots' rows
+    Resolved res;       // the chunk being gathered
 };
 
-// W < 32 class: a task is 32 slots = 32/W rows of one bucket
-__device__ __forceinline__ TaskIn load_narrow(const SpmmArgs &a, int64_t task, int &bcur, int lane, uint64_t pol) {
-    while (bcur + 1 < a.nb_n && __ldg(&a.bk_n[bcur + 1].task_off) <= task) bcur++;
-    const BucketDev *bk = a.bk_n + bcur;
-    const int64_t tin = task - __ldg(&bk->task_off);
-    const int t = __ldg(&bk->t);
-    const int64_t s0 = __ldg(&bk->slot_off) + tin * 32;
-    const int64_t ns = min((int64_t)32, __ldg(&bk->n_slots) - tin * 32);
-    const int64_t nrows = ns >> t;
-    TaskIn x;
-    x.b = bcur;
-    x.c = lane < ns ? ld_stream(a.col + s0 + lane, pol) : -1;
-    x.v = lane < ns ? ld_stream(a.val + s0 + lane, pol) : 0.f;
-    x.tag = lane < nrows ? ld_stream(a.row_tag + __ldg(&bk->row_off) + ((tin * 32) >> t) + lane, pol) : -1;
-    return x;
+__device__ __forceinline__ void cp_async4(void *dst, const void *src, uint64_t pol) {
+    asm volatile("cp.async.ca.shared.global.L2::cache_hint [%0], [%1], 4, %2;" ::"r"(
+                     (uint32_t)__cvta_generic_to_shared(dst)),
+                 "l"(src), "l"(pol)
+                 : "memory");
 }
-
-// W >= 32 class: a task is one CELL row; its first 32 slots are prefetched
-__device__ __forceinline__ TaskIn load_wide(const SpmmArgs &a, int64_t task, int &bcur, int lane, uint64_t pol) {
-    while (bcur + 1 < a.nb_w && __ldg(&a.bk_w[bcur + 1].task_off) <= task) bcur++;
-    const BucketDev *bk = a.bk_w + bcur;
-    const int64_t tin = task - __ldg(&bk->task_off);
-    const int64_t s0 = __ldg(&bk->slot_off) + (tin << __ldg(&bk->t));
-    TaskIn x;
-    x.b = bcur;
-    x.c = ld_stream(a.col + s0 + lane, pol);
-    x.v = ld_stream(a.val + s0 + lane, pol);
-    x.tag = lane == 0 ? ld_stream(a.row_tag + __ldg(&bk->row_off) + tin, pol) : 0;
-    return x;
-}
+__device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
+__device__ __forceinline__ void cp_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
 
 // chunked grid-stride task order: warp w takes tasks [w*CH, w*CH+CH), then
-// advances by nwarps*CH; returns the next task and flags chunk ends
+// advances by nwarps*CH; returns the next task and flags the chunk end
 __device__ __forceinline__ int64_t next_task(int64_t task, int64_t &cs, int64_t round, int64_t n, bool &chunk_end) {
     int64_t tn = task + 1;
     chunk_end = false;
@@ -290,132 +297,231 @@ __device__ __forceinline__ int64_t next_task(int64_t task, int64_t &cs, int64_t 
     return tn;
 }
 
-template <class Cx>
-__device__ __forceinline__ void narrow_loop(const SpmmArgs &a, const Cx &cx0, int2 *sw, int lane, int64_t wid,
-                                            int64_t nw, uint64_t pol) {
-    Cx cx = cx0;
-    constexpr int JT = Cx::L::JT;
-    const int64_t round = nw * kChunk;
-    int64_t cs = wid * kChunk;
-    if (cs >= a.n_tasks_n) return;
-    int bcur = 0;
-    int64_t task = cs;
-    TaskIn cur = load_narrow(a, task, bcur, lane, pol);
-    while (task < a.n_tasks_n) {
-        bool chunk_end;
-        const int64_t tn = next_task(task, cs, round, a.n_tasks_n, chunk_end);
-        TaskIn nxt{};
-        if (tn < a.n_tasks_n) nxt = load_narrow(a, tn, bcur, lane, pol);
-        if (__ballot_sync(kFull, cur.tag >= 0)) {
-            const int t = __ldg(&a.bk_n[cur.b].t);
-            stage<Cx::Gv>(sw, lane, cur.c, cur.v);
-            for (int j0 = 0; j0 < a.J; j0 += JT) {
-                cx.j0 = j0;
-                switch (t) {
-                case 0: narrow_task<Cx, 0>(cx, sw, cur.tag); break;
-                case 1: narrow_task<Cx, 1>(cx, sw, cur.tag); break;
-                case 2: narrow_task<Cx, 2>(cx, sw, cur.tag); break;
-                case 3: narrow_task<Cx, 3>(cx, sw, cur.tag); break;
-                default: narrow_task<Cx, 4>(cx, sw, cur.tag); break;
-                }
-            }
-        }
-        task = tn;
-        cur = nxt;
+// W < 32 class: a task is 32 slots = 32/W rows of one bucket.  Returns t.
+template <int G>
+__device__ __forceinline__ int issue_narrow(const SpmmArgs &a, int64_t task, int &bcur, int lane, uint64_t pol,
+                                            WarpStage &st, int buf) {
+    while (bcur + 1 < a.nb_n && __ldg(&a.bk_n[bcur + 1].task_off) <= task) bcur++;
+    const BucketDev *bk = a.bk_n + bcur;
+    const int64_t tin = task - __ldg(&bk->task_off);
+    const int t = __ldg(&bk->t);
+    const int64_t s0 = __ldg(&bk->slot_off) + tin * 32;
+    const int64_t ns = min((int64_t)32, __ldg(&bk->n_slots) - tin * 32);
+    const int64_t nrows = ns >> t;
+    int2 *dst = &st.slot[buf][stage_pos<G>(lane)];
+    if (lane < ns) {
+        cp_async4(&dst->x, a.col + s0 + lane, pol);
+        cp_async4(&dst->y, a.val + s0 + lane, pol);
+    } else {
+        *dst = make_int2(-1, 0);
     }
+    if (lane < nrows) cp_async4(&st.tag[buf][lane], a.row_tag + __ldg(&bk->row_off) + ((tin * 32) >> t) + lane, pol);
+    else st.tag[buf][lane] = -1;
+    cp_commit();
+    return t;
 }
 
 template <class Cx>
-__device__ __forceinline__ void wide_loop(const SpmmArgs &a, const Cx &cx0, int2 *sw, int lane, int64_t wid,
+__device__ __forceinline__ void narrow_loop(const SpmmArgs &a, const Cx &cx0, WarpStage &st, int lane, int64_t wid,
+                                            int64_t nw, uint64_t pol) {
+    constexpr int G = Cx::Gv, JT = Cx::L::JT;
+    Cx cx = cx0;
+    const int64_t round = nw * kChunk;
+    int64_t cs = wid * kChunk;
+    if (cs >= a.n_tasks_n) return;
+    int bcur = 0, buf = 0;
+    int64_t task = cs;
+    int t = issue_narrow<G>(a, task, bcur, lane, pol, st, 0);
+    while (task < a.n_tasks_n) {
+        bool chunk_end;
+        const int64_t tn = next_task(task, cs, round, a.n_tasks_n, chunk_end);
+        int tnext = 0;
+        if (tn < a.n_tasks_n) tnext = issue_narrow<G>(a, tn, bcur, lane, pol, st, buf ^ 1);
+        else cp_commit();
+        cp_wait1();
+        __syncwarp();
+        const int32_t tag_l = st.tag[buf][lane];
+        if (__ballot_sync(kFull, tag_l >= 0)) {
+            const Resolved &sw = st.res;
+            for (int j0 = 0; j0 < a.J; j0 += JT) {
+                cx.j0 = j0;
+                resolve(cx, st.slot[buf], st.res, lane);
+                switch (t) {
+                case 0: narrow_task<Cx, 0>(cx, sw, tag_l); break;
+                case 1: narrow_task<Cx, 1>(cx, sw, tag_l); break;
+                case 2: narrow_task<Cx, 2>(cx, sw, tag_l); break;
+                case 3: narrow_task<Cx, 3>(cx, sw, tag_l); break;
+                default: narrow_task<Cx, 4>(cx, sw, tag_l); break;
+                }
+            }
+        }
+        __syncwarp();
+        buf ^= 1;
+        task = tn;
+        t = tnext;
+    }
+}
+
+// W >= 32 class: a task is one CELL row = W/32 chunks of 32 slots.
+struct WideCursor {
+    int64_t task;
+    int k, nch;       // chunk within the row, chunks per row
+    int last;         // task is the last of its warp chunk (flush pending runs after it)
+};
+
+template <int G>
+__device__ __forceinline__ void issue_wide(const SpmmArgs &a, const WideCursor &c, int bcur, int lane,
+                                           uint64_t pol, WarpStage &st, int buf) {
+    const BucketDev *bk = a.bk_w + bcur;
+    const int64_t tin = c.task - __ldg(&bk->task_off);
+    const int64_t s = __ldg(&bk->slot_off) + (tin << __ldg(&bk->t)) + 32 * c.k + lane;
+    int2 *dst = &st.slot[buf][stage_pos<G>(lane)];
+    cp_async4(&dst->x, a.col + s, pol);
+    cp_async4(&dst->y, a.val + s, pol);
+    if (c.k == 0 && lane == 0) cp_async4(&st.tag[buf][0], a.row_tag + __ldg(&bk->row_off) + tin, pol);
+    cp_commit();
+}
+
+__device__ __forceinline__ int wide_nch(const SpmmArgs &a, int64_t task, int &bcur) {
+    while (bcur + 1 < a.nb_w && __ldg(&a.bk_w[bcur + 1].task_off) <= task) bcur++;
+    return 1 << (__ldg(&a.bk_w[bcur].t) - 5);
+}
+
+template <class Cx>
+__device__ __forceinline__ void wide_loop(const SpmmArgs &a, const Cx &cx, WarpStage &st, int lane, int64_t wid,
                                           int64_t nw, uint64_t pol) {
     using VT = typename Cx::VT;
-    constexpr int NV = Cx::NVv, G = Cx::Gv, JT = Cx::L::JT;
-    Cx cx = cx0;
-    const bool single_tile = a.J <= JT;  // merge folded rows only without J tiling
+    constexpr int NV = Cx::NVv, G = Cx::Gv;
     const int64_t round = nw * kChunk;
     int64_t cs = wid * kChunk;
     if (cs >= a.n_tasks_w) return;
-    int bcur = 0;
-    int64_t task = cs;
-    TaskIn cur = load_wide(a, task, bcur, lane, pol);
+    int bcur = 0, buf = 0;
+    WideCursor cur{cs, 0, 0, 0};
+    cur.nch = wide_nch(a, cur.task, bcur);
+    int bcur_cur = bcur;
+    issue_wide<G>(a, cur, bcur, lane, pol, st, 0);
     VT acc[NV];
     cx.zero(acc);
-    int32_t pend = -1;  // tag of the run accumulated in acc (-1: none)
+    int32_t pend = -1;      // tag of the run accumulated in acc (-1: none)
+    int32_t row_tag = -1;   // tag of the row being streamed
     bool run_first = false;
-    while (task < a.n_tasks_w) {
-        bool chunk_end;
-        const int64_t tn = next_task(task, cs, round, a.n_tasks_w, chunk_end);
-        TaskIn nxt{};
-        if (tn < a.n_tasks_w) nxt = load_wide(a, tn, bcur, lane, pol);
-        const int32_t tag = __shfl_sync(kFull, cur.tag, 0);
-        if (tag >= 0) {
-            if (pend >= 0 && tag_row(pend) != tag_row(tag)) {  // previous run split off: red
+    while (cur.task < a.n_tasks_w) {
+        // successor chunk
+        WideCursor nx = cur;
+        if (cur.k + 1 < cur.nch) {
+            nx.k = cur.k + 1;
+        } else {
+            bool ce;
+            nx.task = next_task(cur.task, cs, round, a.n_tasks_w, ce);
+            nx.k = 0;
+            cur.last = ce;
+        }
+        int bcur_nx = bcur_cur;
+        if (nx.task < a.n_tasks_w) {
+            if (nx.k == 0) {
+                nx.nch = wide_nch(a, nx.task, bcur);
+                bcur_nx = bcur;
+            }
+            issue_wide<G>(a, nx, bcur_nx, lane, pol, st, buf ^ 1);
+        } else {
+            cp_commit();
+        }
+        cp_wait1();
+        __syncwarp();
+        if (cur.k == 0) {
+            row_tag = st.tag[buf][0];
+            if (row_tag >= 0) {
+                if (pend >= 0 && tag_row(pend) != tag_row(row_tag)) {  // previous run split off: red
+                    cx.reduce_groups(acc);
+                    if (cx.g == 0) cx.write(tag_row(pend), false, acc);
+                    cx.zero(acc);
+                    pend = -1;
+                }
+                if (pend < 0) run_first = (row_tag & 2) != 0;
+            }
+        }
+        if (row_tag >= 0 && __ballot_sync(kFull, st.slot[buf][lane].x >= 0)) {
+            resolve(cx, st.slot[buf], st.res, lane);
+            accum32(cx, st.res, acc);
+        }
+        if (cur.k == cur.nch - 1) {
+            if (row_tag >= 0) {
+                pend = row_tag;
+                if (row_tag & 1) {  // last sub-row of the segment completes the run
+                    cx.reduce_groups(acc);
+                    if (cx.g == 0) cx.write(tag_row(row_tag), run_first && (row_tag & 4), acc);
+                    cx.zero(acc);
+                    pend = -1;
+                }
+            }
+            if (cur.last && pend >= 0) {
                 cx.reduce_groups(acc);
                 if (cx.g == 0) cx.write(tag_row(pend), false, acc);
                 cx.zero(acc);
                 pend = -1;
             }
-            if (pend < 0) run_first = (tag & 2) != 0;
-            const BucketDev *bk = a.bk_w + cur.b;
-            const int t = __ldg(&bk->t);
-            const int64_t s0 = __ldg(&bk->slot_off) + ((task - __ldg(&bk->task_off)) << t);
-            const int64_t W = int64_t(1) << t;
-            for (int j0 = 0; j0 < a.J; j0 += JT) {
-                cx.j0 = j0;
-                stage<G>(sw, lane, cur.c, cur.v);
-                accum32(cx, sw, acc);
-                for (int64_t base = 32; base < W; base += 32) {
-                    const int32_t c_l = ld_stream(a.col + s0 + base + lane, pol);
-                    const float v_l = ld_stream(a.val + s0 + base + lane, pol);
-                    if (__ballot_sync(kFull, c_l >= 0) == 0) break;  // rest is padding
-                    stage<G>(sw, lane, c_l, v_l);
-                    accum32(cx, sw, acc);
-                }
-                if (!single_tile) {  // J tiles: every tile writes its own slice
-                    cx.reduce_groups(acc);
-                    if (cx.g == 0) cx.write(tag_row(tag), tag_whole(tag), acc);
-                    cx.zero(acc);
-                }
-            }
-            if (single_tile) {
-                pend = tag;
-                if (tag & 1) {  // last sub-row of the segment completes the run
-                    cx.reduce_groups(acc);
-                    if (cx.g == 0) cx.write(tag_row(tag), run_first && (tag & 4), acc);
-                    cx.zero(acc);
-                    pend = -1;
-                }
-            }
         }
-        if (chunk_end && pend >= 0) {
-            cx.reduce_groups(acc);
-            if (cx.g == 0) cx.write(tag_row(pend), false, acc);
+        __syncwarp();
+        buf ^= 1;
+        cur = nx;
+        bcur_cur = bcur_nx;
+    }
+}
+
+// J wider than one pass (J > JT): each row is streamed once per J tile,
+// synchronously, and every tile writes its slice (no run merging).
+template <class Cx>
+__device__ __forceinline__ void wide_loop_tiled(const SpmmArgs &a, const Cx &cx0, WarpStage &st, int lane,
+                                                int64_t wid, int64_t nw, uint64_t pol) {
+    using VT = typename Cx::VT;
+    constexpr int NV = Cx::NVv, G = Cx::Gv, JT = Cx::L::JT;
+    Cx cx = cx0;
+    int bcur = 0;
+    for (int64_t task = wid; task < a.n_tasks_w; task += nw) {
+        const int nch = wide_nch(a, task, bcur);
+        const BucketDev *bk = a.bk_w + bcur;
+        const int64_t tin = task - __ldg(&bk->task_off);
+        const int32_t tag = __ldg(a.row_tag + __ldg(&bk->row_off) + tin);
+        if (tag < 0) continue;
+        const int64_t s0 = __ldg(&bk->slot_off) + (tin << __ldg(&bk->t));
+        for (int j0 = 0; j0 < a.J; j0 += JT) {
+            cx.j0 = j0;
+            VT acc[NV];
             cx.zero(acc);
-            pend = -1;
+            for (int k = 0; k < nch; k++) {
+                const int32_t c_l = ld_stream(a.col + s0 + 32 * k + lane, pol);
+                const float v_l = ld_stream(a.val + s0 + 32 * k + lane, pol);
+                if (__ballot_sync(kFull, c_l >= 0) == 0) break;  // rest is padding
+                stage<G>(cx, st.res, lane, c_l, v_l);
+                accum32(cx, st.res, acc);
+            }
+            cx.reduce_groups(acc);
+            if (cx.g == 0) cx.write(tag_row(tag), tag_whole(tag), acc);
         }
-        task = tn;
-        cur = nxt;
     }
 }
 
 // Blocks [0, a.blocks_n) run the W < 32 tasks, the rest the W >= 32 tasks:
-// the two loops share no live state, so each is register-allocated alone.
+// the loops share no live state, so each is register-allocated alone.
 template <int VEC, int G, int NV, bool FULL>
 __global__ void __launch_bounds__(kWarpsPerBlock * 32, kMinBlocks) cell_spmm_kernel(const SpmmArgs a) {
     using Cx = Ctx<VEC, G, NV, FULL>;
     using L = Layout<VEC, G, NV>;
-    __shared__ __align__(16) int2 stage_buf[kWarpsPerBlock][32];
+    __shared__ __align__(16) WarpStage stage_buf[kWarpsPerBlock];
     const int lane = threadIdx.x & 31;
-    int2 *sw = stage_buf[threadIdx.x >> 5];
+    WarpStage &st = stage_buf[threadIdx.x >> 5];
     const uint64_t pol = policy_evict_first();
     const Cx cx{a.B, a.ldb, a.C, a.ldc, a.J, 0, lane / L::LPR, lane % L::LPR, pol};
     const int w = threadIdx.x >> 5;
-    if ((int)blockIdx.x < a.blocks_n)
-        narrow_loop(a, cx, sw, lane, (int64_t)blockIdx.x * kWarpsPerBlock + w, (int64_t)a.blocks_n * kWarpsPerBlock,
+    if ((int)blockIdx.x < a.blocks_n) {
+        narrow_loop(a, cx, st, lane, (int64_t)blockIdx.x * kWarpsPerBlock + w, (int64_t)a.blocks_n * kWarpsPerBlock,
                     pol);
-    else
-        wide_loop(a, cx, sw, lane, (int64_t)(blockIdx.x - a.blocks_n) * kWarpsPerBlock + w,
-                  (int64_t)(gridDim.x - a.blocks_n) * kWarpsPerBlock, pol);
+    } else {
+        const int64_t wid = (int64_t)(blockIdx.x - a.blocks_n) * kWarpsPerBlock + w;
+        const int64_t nw = (int64_t)(gridDim.x - a.blocks_n) * kWarpsPerBlock;
+        if (a.J <= L::JT) wide_loop(a, cx, st, lane, wid, nw, pol);
+        else wide_loop_tiled(a, cx, st, lane, wid, nw, pol);
+    }
 }
 
 // Algorithm 1 on the GPU straight from CSR: one warp per row, same lane layout.
@@ -427,9 +533,9 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32)
     using Cx = Ctx<VEC, G, NV, FULL>;
     using VT = typename Cx::VT;
     using L = Layout<VEC, G, NV>;
-    __shared__ __align__(16) int2 stage_buf[kWarpsPerBlock][32];
+    __shared__ __align__(16) Resolved stage_buf[kWarpsPerBlock];
     const int lane = threadIdx.x & 31;
-    int2 *sw = stage_buf[threadIdx.x >> 5];
+    Resolved &sw = stage_buf[threadIdx.x >> 5];
     const int64_t gwarp = (int64_t)blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5);
     const int64_t nwarps = (int64_t)gridDim.x * kWarpsPerBlock;
     const uint64_t pol = policy_evict_first();
@@ -442,7 +548,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32)
             cx.zero(acc);
             for (int64_t base = rb; base < re; base += 32) {
                 const bool in = base + lane < re;
-                stage<G>(sw, lane, in ? ld_stream(col + base + lane, pol) : -1,
+                stage<G>(cx, sw, lane, in ? ld_stream(col + base + lane, pol) : -1,
                          in ? ld_stream(val + base + lane, pol) : 0.f);
                 accum32(cx, sw, acc);
             }
