@@ -189,40 +189,68 @@ __global__ void __launch_bounds__(1024) tile_scan_kernel(long long *__restrict__
 }
 
 constexpr int kSlotThreads = 256;
+constexpr int kSlotILP = 4;  // independent slots per thread per iteration
 constexpr int kMaxSmemBuckets = 2048;
 
+// One thread per slot (kSlotILP slots in flight per thread): bucket of the
+// slot (binary search over the bucket slot offsets in shared memory), its
+// CELL row and position w in the row; real slots copy colInd/val from the
+// CSR position src_pos[row] + w, the rest get the padding (-1, +0.0f).
 __global__ void __launch_bounds__(kSlotThreads)
     slot_fill_kernel(const int32_t *__restrict__ col, const float *__restrict__ val,
                      const BucketDev *__restrict__ bk, int nb, int64_t n_slots, const int64_t *__restrict__ src_pos,
                      const int32_t *__restrict__ src_cnt, int32_t *__restrict__ col_out,
                      float *__restrict__ val_out) {
     __shared__ int64_t soff[kMaxSmemBuckets];
-    for (int q = threadIdx.x; q < nb; q += blockDim.x) soff[q] = bk[q].slot_off;
+    __shared__ int64_t roff[kMaxSmemBuckets];
+    __shared__ int32_t tt[kMaxSmemBuckets];
+    for (int q = threadIdx.x; q < nb; q += blockDim.x) {
+        soff[q] = bk[q].slot_off;
+        roff[q] = bk[q].row_off;
+        tt[q] = bk[q].t;
+    }
     __syncthreads();
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    int b = 0;
-    for (int64_t s = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; s < n_slots; s += stride) {
-        // bucket of slot s: last b with soff[b] <= s (monotone in s for this thread)
-        int lo = b, hi = nb - 1;
-        while (lo < hi) {
-            int mid = (lo + hi + 1) >> 1;
-            if (soff[mid] <= s) lo = mid;
-            else hi = mid - 1;
+    for (int64_t s0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; s0 < n_slots; s0 += stride * kSlotILP) {
+        int64_t pos[kSlotILP];
+        int32_t cnt[kSlotILP], w[kSlotILP];
+#pragma unroll
+        for (int k = 0; k < kSlotILP; k++) {
+            const int64_t s = s0 + k * stride;
+            cnt[k] = 0;
+            w[k] = 1;
+            pos[k] = 0;
+            if (s < n_slots) {
+                int lo = 0, hi = nb - 1;  // last bucket with soff <= s
+                while (lo < hi) {
+                    const int mid = (lo + hi + 1) >> 1;
+                    if (soff[mid] <= s) lo = mid;
+                    else hi = mid - 1;
+                }
+                const int t = tt[lo];
+                const int64_t rel = s - soff[lo];
+                const int64_t r = roff[lo] + (rel >> t);
+                w[k] = (int32_t)(rel & ((int64_t(1) << t) - 1));
+                cnt[k] = __ldg(src_cnt + r);
+                pos[k] = __ldg(src_pos + r);
+            }
         }
-        b = lo;
-        const int t = bk[b].t;
-        const int64_t rel = s - soff[b];
-        const int64_t r = bk[b].row_off + (rel >> t);
-        const int64_t w = rel & ((int64_t(1) << t) - 1);
-        int32_t c = -1;
-        float v = 0.0f;
-        if (w < src_cnt[r]) {
-            const int64_t pos = src_pos[r] + w;
-            c = col[pos];
-            v = val[pos];
+        int32_t c[kSlotILP];
+        float v[kSlotILP];
+#pragma unroll
+        for (int k = 0; k < kSlotILP; k++) {
+            const bool real = w[k] < cnt[k];
+            c[k] = real ? __ldg(col + pos[k] + w[k]) : -1;
+            v[k] = real ? __ldg(val + pos[k] + w[k]) : 0.0f;
         }
-        col_out[s] = c;
-        val_out[s] = v;
+#pragma unroll
+        for (int k = 0; k < kSlotILP; k++) {
+            const int64_t s = s0 + k * stride;
+            if (s < n_slots) {
+                __stcs(col_out + s, c[k]);
+                __stcs(val_out + s, v[k]);
+            }
+        }
     }
 }
 
@@ -282,7 +310,7 @@ cudaError_t launch_slot_fill(const lf_csr &A, const BucketDev *d_buckets, int nb
                              const BuildScratch &sc, int32_t *col_out, float *val_out, cudaStream_t s) {
     if (n_slots == 0) return cudaSuccess;
     if (nb > kMaxSmemBuckets) return cudaErrorInvalidValue;
-    slot_fill_kernel<<<grid_for(n_slots, kSlotThreads), kSlotThreads, 0, s>>>(
+    slot_fill_kernel<<<grid_for((n_slots + kSlotILP - 1) / kSlotILP, kSlotThreads), kSlotThreads, 0, s>>>(
         A.col_ind, A.val, d_buckets, nb, n_slots, sc.src_pos, sc.src_cnt, col_out, val_out);
     return cudaGetLastError();
 }

@@ -5,10 +5,10 @@
 //   H[p][t]  segment count,  F[p][t] = sum_{t0 >= t} ceil(l / 2^t)  (fold rows),
 //   Unat[p][t], Utop[p][t]   the |set(Ind)| terms of eq. 7
 // plus the Table 2 row-length statistics.  Three passes:
-//   stats_rows_kernel   one thread per row: segments, H, F (warp-aggregated
-//                       with REDUX), features; writes t0 of every segment
-//   stats_mark_kernel   nnz-balanced: column c of segment (i,p) sets bit t0 of
-//                       a per-column mask M[c] (partition of c is c / S)
+//   stats_rows_kernel   one thread per row: segments, H, F (warp-aggregated),
+//                       features; t0 of every segment -> t0seg
+//   stats_mark_kernel   nnz-balanced: every nonzero sets bit t0 of its segment
+//                       in the per-column mask M[c] (partition of c is c / S)
 //   stats_cols_kernel   one thread per column: Unat[p][t] = #{c : bit t},
 //                       Utop[p][t] = #{c : highest bit >= t} (warp-aggregated)
 #include "../lf_internal.cuh"
@@ -18,8 +18,6 @@ namespace lf {
 namespace {
 
 constexpr int kThreads = 256;
-constexpr int kMarkPerThread = 16;
-constexpr int kMarkTile = kThreads * kMarkPerThread;
 constexpr unsigned kFull = 0xffffffffu;
 constexpr uint8_t kEmpty = 0xFF;
 
@@ -40,10 +38,27 @@ __device__ __forceinline__ unsigned long long warp_sum_u31(unsigned v) {
     return ((unsigned long long)hi << 16) + lo;
 }
 
+// Pass 1 -- one thread per row: segments of the row in every partition, their
+// natural bucket t0 (written to t0seg[i*P+p]), the H / F histograms
+// (warp-aggregated: __match_any_sync for H, REDUX for F) and the Table 2
+// row-length statistics.
+#ifndef LF_MARK_TILE
+#define LF_MARK_TILE 4096
+#endif
+constexpr int kMarkTile = LF_MARK_TILE;
+#ifndef LF_MARK_L1
+#define LF_MARK_L1 0
+#endif
+#ifndef LF_MARK_MATCH
+#define LF_MARK_MATCH 0
+#endif  // nonzeros per block of the marking pass
+
 __global__ void __launch_bounds__(kThreads) stats_rows_kernel(const int64_t *__restrict__ row_ptr,
                                                               const int32_t *__restrict__ col, int64_t n_rows,
                                                               int64_t S, int P, StatsDev *st,
-                                                              uint8_t *__restrict__ t0seg) {
+                                                              uint8_t *__restrict__ t0seg,
+                                                              int64_t *__restrict__ tile_row,
+                                                              int64_t *__restrict__ tile_pos) {
     extern __shared__ unsigned long long sh[];  // H_s[P][32], F_s[P][32]
     unsigned long long *H_s = sh, *F_s = sh + P * kMaxT;
     for (int q = threadIdx.x; q < 2 * P * kMaxT; q += blockDim.x) sh[q] = 0;
@@ -58,7 +73,16 @@ __global__ void __launch_bounds__(kThreads) stats_rows_kernel(const int64_t *__r
         if (active) {
             rb = row_ptr[i];
             re = row_ptr[i + 1];
-            unsigned long long len = (unsigned long long)(re - rb);
+            const unsigned long long len = (unsigned long long)(re - rb);
+            // merge-path tiles over items = (row ends, nonzeros): row i owns items
+            // [rb + i, re + i + 1); tile T starts at item T * kMarkTile, inside
+            // row tile_row[T] at position tile_pos[T] (relative to row_ptr[0])
+            const int64_t base = row_ptr[0];
+            const int64_t b_item = rb - base + i, e_item = re - base + i + 1;
+            for (int64_t T = (b_item + kMarkTile - 1) / kMarkTile; T * kMarkTile < e_item; T++) {
+                tile_row[T] = i;
+                tile_pos[T] = min(T * kMarkTile - i, re - base);
+            }
             mn = min(mn, len);
             mx = max(mx, len);
             sum += len;
@@ -70,18 +94,15 @@ __global__ void __launch_bounds__(kThreads) stats_rows_kernel(const int64_t *__r
             const int64_t l = e - b;
             const int t0 = l > 0 ? ceil_log2_i64(l) : kMaxT;
             if (active) t0seg[i * P + p] = l > 0 ? (uint8_t)t0 : kEmpty;
-            // H: one shared atomic per distinct t0 in the warp
             const unsigned peers = __match_any_sync(kFull, t0);
             if (t0 < kMaxT && (peers & ((1u << lane) - 1u)) == 0)
                 atomicAdd(&H_s[p * kMaxT + t0], (unsigned long long)__popc(peers));
-            // F[t] for t <= t0 (REDUX per level up to the warp's largest t0)
             const int tmax = __reduce_max_sync(kFull, l > 0 ? (unsigned)t0 : 0u);
-            const bool any = __any_sync(kFull, l > 0);
-            if (any) {
+            if (__any_sync(kFull, l > 0)) {
                 for (int t = 0; t <= tmax; t++) {
-                    unsigned v = (l > 0 && t <= t0) ? (unsigned)((l + (int64_t(1) << t) - 1) >> t) : 0u;
-                    unsigned long long s = warp_sum_u31(v);
-                    if (lane == 0 && s) atomicAdd(&F_s[p * kMaxT + t], s);
+                    const unsigned v = (l > 0 && t <= t0) ? (unsigned)((l + (int64_t(1) << t) - 1) >> t) : 0u;
+                    const unsigned long long sv = warp_sum_u31(v);
+                    if (lane == 0 && sv) atomicAdd(&F_s[p * kMaxT + t], sv);
                 }
             }
             b = e;
@@ -106,66 +127,122 @@ __global__ void __launch_bounds__(kThreads) stats_rows_kernel(const int64_t *__r
     }
 }
 
-// nnz-balanced column marking.  Every lane owns kMarkPerThread consecutive
-// positions: one binary search in row_ptr finds the row of its first
-// position, then rows advance as positions cross row_ptr boundaries.
-// Power-law inputs send a large share of all nonzeros to a few hot columns
-// whose mask words share L2 lines, so a per-block direct-mapped filter in
-// shared memory ((col << 32) | bits already set globally, one 64-bit word per
-// slot, updated with whole-word stores so a (col, bits) pair is always
-// consistent) drops repeated (col, bit) pairs before they reach L2.
-constexpr int kFilter = 4096;
+// Pass 2 -- column marking over merge-path tiles: tile T holds kMarkTile
+// items of the sequence (row ends, nonzeros), so at most kMarkTile rows and
+// kMarkTile nonzeros, whatever the row lengths (pass 1 wrote each tile's
+// first row and position).  The block ORs bit t0 of each nonzero's segment
+// into the mask word of its column.  Row of every nonzero: the block counts
+// the rows starting at each tile position (empty rows included) and an
+// inclusive block scan of those counts maps position -> row (one LDS per
+// nonzero).  Nonzeros are read coalesced, kMarkTile / kThreads per thread in
+// one batch so the dependent loads overlap, and every (column, bits) pair
+// goes out as a fire-and-forget RED after a warp-level merge of equal columns.
+// The mask word of column c lives at slot hslot(c) = (c * odd) mod 2^m, a
+// bijection on [0, 2^m), 2^m >= K: columns that are hot together on power-law
+// inputs (small indices, few set bits) land on different L2 lines and slices.
+__device__ __forceinline__ uint32_t hslot(int32_t c, uint32_t kmask) { return ((uint32_t)c * 0x9E3779B1u) & kmask; }
 
 __global__ void __launch_bounds__(kThreads) stats_mark_kernel(const int64_t *__restrict__ row_ptr,
                                                               const int32_t *__restrict__ col, int64_t n_rows,
                                                               int64_t S, int P,
                                                               const uint8_t *__restrict__ t0seg,
-                                                              uint32_t *__restrict__ mask) {
-    __shared__ unsigned long long filt[kFilter];
-    for (int q = threadIdx.x; q < kFilter; q += blockDim.x) filt[q] = ~0ull;  // col field 0xFFFFFFFF: empty
-    __syncthreads();
+                                                              const int64_t *__restrict__ tile_row,
+                                                              const int64_t *__restrict__ tile_pos, int64_t n_tiles,
+                                                              uint32_t *__restrict__ mask, uint32_t kmask) {
+    __shared__ int32_t cnt[kMarkTile];     // rows starting at a tile position -> inclusive scan
+    __shared__ uint8_t rt0[kMarkTile + 1]; // t0 of the tile's rows (P == 1)
+    __shared__ int32_t wsum[kThreads / 32];
+    constexpr int K = kMarkTile / kThreads;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    for (int q = threadIdx.x; q < kMarkTile; q += blockDim.x) cnt[q] = 0;
     const int64_t base = row_ptr[0];
-    const int64_t nnz = row_ptr[n_rows] - base;
-    const int64_t stride = (int64_t)gridDim.x * blockDim.x * kMarkPerThread;
-    for (int64_t q0 = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) * kMarkPerThread; q0 < nnz; q0 += stride) {
-        // row of position q0: last r with row_ptr[r] - base <= q0
-        int64_t lo = 0, hi = n_rows - 1;
-        while (lo < hi) {
-            const int64_t m = (lo + hi + 1) >> 1;
-            if (__ldg(row_ptr + m) - base <= q0) lo = m;
-            else hi = m - 1;
-        }
-        int64_t r = lo;
-        int64_t rend = __ldg(row_ptr + r + 1) - base;
-        int32_t c[kMarkPerThread];
-        uint32_t bit[kMarkPerThread];
+    const int64_t T = blockIdx.x;
+    const int64_t rlo = tile_row[T];
+    const int64_t qa = base + tile_pos[T];
+    const int64_t rhi = T + 1 < n_tiles ? tile_row[T + 1] : n_rows - 1;
+    const int64_t qb = T + 1 < n_tiles ? base + tile_pos[T + 1] : row_ptr[n_rows];
+    __syncthreads();
+    {
+        constexpr int RU = 8;  // independent row_ptr loads in flight per thread
+        for (int64_t r0 = rlo + threadIdx.x; r0 <= rhi; r0 += (int64_t)blockDim.x * RU) {
+            int64_t sr[RU], er[RU];
 #pragma unroll
-        for (int k = 0; k < kMarkPerThread; k++) {
-            const int64_t q = q0 + k;
-            c[k] = -1;
-            bit[k] = 0;
-            if (q < nnz) {
-                while (q >= rend) rend = __ldg(row_ptr + (++r) + 1) - base;
-                c[k] = __ldg(col + base + q);
-                const int p = P == 1 ? 0 : (int)(c[k] / S);
-                bit[k] = 1u << __ldg(t0seg + r * P + p);
+            for (int u = 0; u < RU; u++) {
+                const int64_t r = r0 + (int64_t)u * blockDim.x;
+                sr[u] = r <= rhi ? __ldg(row_ptr + r) - qa : 0;
+                er[u] = r <= rhi ? __ldg(row_ptr + r + 1) - qa : 0;
+            }
+#pragma unroll
+            for (int u = 0; u < RU; u++) {
+                const int64_t r = r0 + (int64_t)u * blockDim.x;
+                if (r > rhi) break;
+                if (P == 1) rt0[r - rlo] = (uint8_t)ceil_log2_i64(max(er[u] - sr[u], (int64_t)1));
+                if (r > rlo && sr[u] < qb - qa) atomicAdd(&cnt[sr[u]], 1);
             }
         }
-#pragma unroll
-        for (int k = 0; k < kMarkPerThread; k++) {
-            if (c[k] < 0) continue;
-            const int slot = c[k] & (kFilter - 1);
-            const unsigned long long f = filt[slot];
-            const bool same = (uint32_t)(f >> 32) == (uint32_t)c[k];
-            if (same && ((uint32_t)f & bit[k])) continue;
-            atomicOr(mask + c[k], bit[k]);
-            filt[slot] = ((unsigned long long)(uint32_t)c[k] << 32) | (same ? ((uint32_t)f | bit[k]) : bit[k]);
-        }
     }
+    __syncthreads();
+    {  // inclusive scan of cnt, conflict-free: warp w scans its 512 entries in
+       // 32-wide chunks (shuffles), then adds the totals of the warps before it
+        constexpr int PER_WARP = kMarkTile / (kThreads / 32);
+        int32_t carry = 0;
+        for (int j = 0; j < PER_WARP; j += 32) {
+            const int idx = warp * PER_WARP + j + lane;
+            int32_t x = cnt[idx];
+            for (int o = 1; o < 32; o <<= 1) {
+                const int32_t y = __shfl_up_sync(kFull, x, o);
+                if (lane >= o) x += y;
+            }
+            cnt[idx] = x + carry;
+            carry += __shfl_sync(kFull, x, 31);
+        }
+        if (lane == 0) wsum[warp] = carry;
+        __syncthreads();
+        int32_t off = 0;
+        for (int w = 0; w < warp; w++) off += wsum[w];
+        if (off)
+            for (int j = lane; j < PER_WARP; j += 32) cnt[warp * PER_WARP + j] += off;
+    }
+    __syncthreads();
+    int32_t c[K];
+    uint32_t bit[K];
+#pragma unroll
+    for (int k = 0; k < K; k++) {
+        const int64_t q = qa + k * kThreads + threadIdx.x;
+        c[k] = q < qb ? __ldg(col + q) : -1;
+    }
+#pragma unroll
+    for (int k = 0; k < K; k++) {
+        bit[k] = 0;
+        if (c[k] < 0) continue;
+        const int rr = cnt[k * kThreads + threadIdx.x];
+        if (P == 1) bit[k] = 1u << rt0[rr];
+        else bit[k] = 1u << __ldg(t0seg + (rlo + rr) * P + (int)(c[k] / S));
+    }
+    // L2 atomics are expensive (a few tens of G/s chip-wide) and most
+    // (column, bit) pairs are already set, so: keep one lane per distinct
+    // (column, bit) of the warp (__match_any_sync), read every mask word with one unconditional
+    // batch of L2 loads, and issue a RED only for bits still missing.
+    uint32_t h[K], have[K];
+#pragma unroll
+    for (int k = 0; k < K; k++) {
+#if LF_MARK_MATCH
+        const unsigned long long key = ((unsigned long long)(uint32_t)c[k] << 32) | bit[k];
+        const unsigned peers = __match_any_sync(kFull, key);
+        const bool leader = c[k] >= 0 && (peers & ((1u << lane) - 1u)) == 0;
+        bit[k] = leader ? bit[k] : 0u;
+#endif
+        h[k] = c[k] >= 0 ? hslot(c[k], kmask) : 0u;
+    }
+#pragma unroll
+    for (int k = 0; k < K; k++) have[k] = LF_MARK_L1 ? mask[h[k]] : __ldcg(mask + h[k]);
+#pragma unroll
+    for (int k = 0; k < K; k++)
+        if ((have[k] & bit[k]) != bit[k]) atomicOr(mask + h[k], bit[k]);
 }
 
 __global__ void __launch_bounds__(kThreads) stats_cols_kernel(const uint32_t *__restrict__ mask, int64_t n_cols,
-                                                              int64_t S, int P, StatsDev *st) {
+                                                              int64_t S, int P, StatsDev *st, uint32_t kmask) {
     extern __shared__ unsigned long long sh[];  // Un_s[P][32], Ut_s[P][32]
     unsigned long long *Un_s = sh, *Ut_s = sh + P * kMaxT;
     for (int q = threadIdx.x; q < 2 * P * kMaxT; q += blockDim.x) sh[q] = 0;
@@ -174,7 +251,7 @@ __global__ void __launch_bounds__(kThreads) stats_cols_kernel(const uint32_t *__
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < n_cols; base += stride) {
         const int64_t c = base + threadIdx.x;
-        const uint32_t m = c < n_cols ? mask[c] : 0u;
+        const uint32_t m = c < n_cols ? __ldg(mask + hslot((int32_t)c, kmask)) : 0u;
         const int p = c < n_cols ? (int)(c / S) : -1;
         const int hb = m ? 31 - __clz(m) : -1;
         // columns of one warp may straddle a partition boundary: group by p
@@ -214,24 +291,38 @@ int num_sms() {
 
 }  // namespace
 
+size_t stats_scratch_bytes(int64_t n_rows, int64_t nnz, int P) {
+    return (((size_t)n_rows * P + 15) & ~size_t(15)) + (size_t)((nnz + n_rows + kMarkTile - 1) / kMarkTile + 1) * 16;
+}
+
+uint32_t mask_slots(int64_t n_cols) {
+    uint64_t m = 1;
+    while ((int64_t)m < n_cols) m <<= 1;
+    return (uint32_t)m;
+}
+
 cudaError_t launch_stats(const lf_csr &A, int P, StatsDev *d_stats, uint32_t *d_colmask, uint8_t *d_t0seg,
                          cudaStream_t s) {
     const int64_t S = A.n_cols > 0 ? (A.n_cols + P - 1) / P : 1;
-    const size_t smem = 2 * (size_t)P * kMaxT * sizeof(unsigned long long);
+    const size_t hist = 2 * (size_t)P * kMaxT * sizeof(unsigned long long);
     if (A.n_rows > 0) {
-        int64_t want = (A.n_rows + kThreads - 1) / kThreads;
-        int grid = (int)std::min<int64_t>(want, (int64_t)num_sms() * 8);
-        stats_rows_kernel<<<grid, kThreads, smem, s>>>(A.row_ptr, A.col_ind, A.n_rows, S, P, d_stats, d_t0seg);
-        if (A.nnz > 0) {
-            int64_t tiles = (A.nnz + kMarkTile - 1) / kMarkTile;
-            int g2 = (int)std::min<int64_t>(tiles, (int64_t)num_sms() * 16);
-            stats_mark_kernel<<<g2, kThreads, 0, s>>>(A.row_ptr, A.col_ind, A.n_rows, S, P, d_t0seg, d_colmask);
-        }
+        const int64_t want = (A.n_rows + kThreads - 1) / kThreads;
+        const int grid = (int)std::min<int64_t>(want, (int64_t)num_sms() * 8);
+        const int64_t tiles = (A.nnz + A.n_rows + kMarkTile - 1) / kMarkTile;
+        if (tiles > 0x7fffffff) return cudaErrorInvalidValue;
+        int64_t *tile_row = reinterpret_cast<int64_t *>(d_t0seg + (((size_t)A.n_rows * P + 15) & ~size_t(15)));
+        int64_t *tile_pos = tile_row + tiles;
+        stats_rows_kernel<<<grid, kThreads, hist, s>>>(A.row_ptr, A.col_ind, A.n_rows, S, P, d_stats, d_t0seg,
+                                                        tile_row, tile_pos);
+        if (A.nnz > 0)
+            stats_mark_kernel<<<(unsigned)tiles, kThreads, 0, s>>>(A.row_ptr, A.col_ind, A.n_rows, S, P, d_t0seg,
+                                                                    tile_row, tile_pos, tiles, d_colmask,
+                                                                    mask_slots(A.n_cols) - 1);
     }
     if (A.n_cols > 0) {
-        int64_t want = (A.n_cols + kThreads - 1) / kThreads;
-        int grid = (int)std::min<int64_t>(want, (int64_t)num_sms() * 8);
-        stats_cols_kernel<<<grid, kThreads, smem, s>>>(d_colmask, A.n_cols, S, P, d_stats);
+        const int64_t want = (A.n_cols + kThreads - 1) / kThreads;
+        const int grid = (int)std::min<int64_t>(want, (int64_t)num_sms() * 8);
+        stats_cols_kernel<<<grid, kThreads, hist, s>>>(d_colmask, A.n_cols, S, P, d_stats, mask_slots(A.n_cols) - 1);
     }
     return cudaGetLastError();
 }

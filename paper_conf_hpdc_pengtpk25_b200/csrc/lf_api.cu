@@ -168,11 +168,12 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
     LF_CUDA(cudaMemsetAsync(d_st, 0, sizeof(lf::StatsDev), s));
     LF_CUDA(cudaMemsetAsync(&d_st->len_min, 0xFF, sizeof(unsigned long long), s));
     if (A->n_cols > 0) {
-        LF_CUDA(cudaMallocAsync(&d_mask, (size_t)A->n_cols * sizeof(uint32_t), s));
-        LF_CUDA(cudaMemsetAsync(d_mask, 0, (size_t)A->n_cols * sizeof(uint32_t), s));
+        const size_t words = lf::mask_slots(A->n_cols);
+        LF_CUDA(cudaMallocAsync(&d_mask, words * sizeof(uint32_t), s));
+        LF_CUDA(cudaMemsetAsync(d_mask, 0, words * sizeof(uint32_t), s));
     }
     uint8_t *d_t0 = nullptr;
-    if (A->n_rows > 0) LF_CUDA(cudaMallocAsync(&d_t0, (size_t)A->n_rows * P, s));
+    if (A->n_rows > 0) LF_CUDA(cudaMallocAsync(&d_t0, lf::stats_scratch_bytes(A->n_rows, A->nnz, P), s));
     LF_CUDA(lf::launch_stats(*A, P, d_st, d_mask, d_t0, s));
     std::vector<lf::StatsDev> h(1);
     LF_CUDA(cudaMemcpyAsync(h.data(), d_st, sizeof(lf::StatsDev), cudaMemcpyDeviceToHost, s));

@@ -46,6 +46,8 @@ struct StatsDev {
 };
 
 // ---- launchers (kernels in csrc/kernels/*.cu) ----
+uint32_t mask_slots(int64_t n_cols);  // words of the column-mask array (power of two >= K)
+size_t stats_scratch_bytes(int64_t n_rows, int64_t nnz, int P);  // t0 per segment + tile -> row map
 cudaError_t launch_stats(const lf_csr &A, int P, StatsDev *d_stats, uint32_t *d_colmask, uint8_t *d_t0seg,
                          cudaStream_t s);
 
