@@ -64,7 +64,7 @@ __global__ void __launch_bounds__(kThreads)
                   const int8_t *__restrict__ e_of_p, int n_tiles, long long *__restrict__ tile_cnt,
                   const long long *__restrict__ key_row_off, int32_t *__restrict__ row_cnt,
                   int32_t *__restrict__ row_ind, int32_t *__restrict__ row_tag, int64_t *__restrict__ src_pos,
-                  int32_t *__restrict__ src_cnt) {
+                  int32_t *__restrict__ src_cnt, uint8_t *__restrict__ row_mode) {
     __shared__ long long warp_tot[kWarps][kMaxT];
     const int tile = blockIdx.x, p = blockIdx.y;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -116,9 +116,13 @@ __global__ void __launch_bounds__(kThreads)
         if (key != kNoKey) {
             pos = key_row_off[p * kMaxT + key] + tile_cnt[((int64_t)p * kMaxT + key) * n_tiles + tile] +
                   warp_tot[warp][key] + rank;
-            // (i << 3) | S << 2 | F << 1 | L  (cell_spmm.cu): S = this segment holds
-            // all of row i's CELL rows; F / L are added per sub-row below
-            tag = (int32_t)((i << 3) | (row_cnt[i] == n_sub ? 4 : 0));
+            // (i << 3) | S << 2 | F << 1 | L  (cell_spmm.cu): S = the row is "whole":
+            // this segment holds all of row i's CELL rows and one warp sums them
+            // (single CELL row, or a run of <= kMaxRun rows in a wide bucket);
+            // F / L mark the first / last sub-row and are added below
+            const bool whole = row_cnt[i] == n_sub && (n_sub == 1 || (key >= 5 && n_sub <= kMaxRun));
+            tag = (int32_t)((i << 3) | (whole ? 4 : 0));
+            row_mode[i] = whole ? (n_sub == 1 ? kRowPlain : kRowRun) : kRowRed;
         }
         const int64_t W = int64_t(1) << (key == kNoKey ? 0 : key);
         if (n_sub <= 32) {
@@ -254,6 +258,37 @@ __global__ void __launch_bounds__(kSlotThreads)
     }
 }
 
+// run_bound[x] for every wide task x (0..n): offset to the first task >= x
+// that starts a run (F), is a padding row, or belongs to a row written with
+// atomics (!S); n counts as a bound.  A whole run (<= kMaxRun <= 32 CELL
+// rows) never straddles two work claims whose ends are aligned this way.
+// One warp per 32 positions, over a 64-task window of boundary flags.
+__device__ __forceinline__ bool is_bound(const BucketDev *__restrict__ bk, int nb, int64_t n,
+                                         const int32_t *__restrict__ tag, int64_t p) {
+    if (p >= n) return true;
+    int lo = 0, hi = nb - 1;  // bucket of task p
+    while (lo < hi) {
+        const int mid = (lo + hi + 1) >> 1;
+        if (bk[mid].task_off <= p) lo = mid;
+        else hi = mid - 1;
+    }
+    const int32_t tg = tag[bk[lo].row_off + (p - bk[lo].task_off)];
+    return tg < 0 || (tg & 2) || !(tg & 4);
+}
+
+__global__ void run_bounds_kernel(const BucketDev *__restrict__ bk, int nb, int64_t n, const int32_t *__restrict__ tag,
+                                  uint8_t *__restrict__ out, int64_t n_out) {
+    const int lane = threadIdx.x & 31;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; w * 32 < n_out; w += nw) {
+        const int64_t x0 = w * 32;
+        const unsigned m1 = __ballot_sync(0xffffffffu, is_bound(bk, nb, n, tag, x0 + lane));
+        const unsigned m2 = __ballot_sync(0xffffffffu, is_bound(bk, nb, n, tag, x0 + 32 + lane));
+        const unsigned long long m = ((unsigned long long)m2 << 32 | m1) >> lane;  // bit 0 = position x0 + lane
+        if (x0 + lane < n_out) out[x0 + lane] = (uint8_t)(m ? min(__ffsll((long long)m) - 1, 32) : 32);
+    }
+}
+
 __global__ void validate_kernel(const int64_t *__restrict__ row_ptr, const int32_t *__restrict__ col, int64_t n_rows,
                                 int64_t n_cols, int *flag) {
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
@@ -287,7 +322,7 @@ cudaError_t launch_bucket_count(const lf_csr &A, int P, const int8_t *e, const B
     if (A.n_rows == 0) return cudaSuccess;
     dim3 grid(sc.n_tiles, P);
     bucket_kernel<0><<<grid, kThreads, 0, s>>>(A.row_ptr, sc.seg_rel, A.n_rows, P, e, sc.n_tiles, sc.tile_cnt,
-                                                nullptr, row_cnt, nullptr, nullptr, nullptr, nullptr);
+                                                nullptr, row_cnt, nullptr, nullptr, nullptr, nullptr, nullptr);
     return cudaGetLastError();
 }
 
@@ -297,12 +332,13 @@ cudaError_t launch_tile_scan(int P, const BuildScratch &sc, cudaStream_t s) {
 }
 
 cudaError_t launch_bucket_place(const lf_csr &A, int P, const int8_t *e, const BuildScratch &sc,
-                                const int32_t *row_cnt, int32_t *row_ind, int32_t *row_tag, cudaStream_t s) {
+                                const int32_t *row_cnt, int32_t *row_ind, int32_t *row_tag, uint8_t *row_mode,
+                                cudaStream_t s) {
     if (A.n_rows == 0) return cudaSuccess;
     dim3 grid(sc.n_tiles, P);
     bucket_kernel<1><<<grid, kThreads, 0, s>>>(A.row_ptr, sc.seg_rel, A.n_rows, P, e, sc.n_tiles, sc.tile_cnt,
                                                 sc.key_row_off, const_cast<int32_t *>(row_cnt), row_ind, row_tag,
-                                                sc.src_pos, sc.src_cnt);
+                                                sc.src_pos, sc.src_cnt, row_mode);
     return cudaGetLastError();
 }
 
@@ -312,6 +348,14 @@ cudaError_t launch_slot_fill(const lf_csr &A, const BucketDev *d_buckets, int nb
     if (nb > kMaxSmemBuckets) return cudaErrorInvalidValue;
     slot_fill_kernel<<<grid_for((n_slots + kSlotILP - 1) / kSlotILP, kSlotThreads), kSlotThreads, 0, s>>>(
         A.col_ind, A.val, d_buckets, nb, n_slots, sc.src_pos, sc.src_cnt, col_out, val_out);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_run_bounds(const BucketDev *bk_w, int nb_w, int64_t n_tasks_w, const int32_t *row_tag,
+                              uint8_t *run_bound, cudaStream_t s) {
+    const int64_t n_out = n_tasks_w + 1;
+    if (nb_w == 0) return cudaMemsetAsync(run_bound, 0, (size_t)n_out, s);
+    run_bounds_kernel<<<grid_for(n_out, 256), 256, 0, s>>>(bk_w, nb_w, n_tasks_w, row_tag, run_bound, n_out);
     return cudaGetLastError();
 }
 

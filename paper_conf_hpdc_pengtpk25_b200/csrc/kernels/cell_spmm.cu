@@ -29,13 +29,20 @@
 // segment holds all of the row's CELL rows; -1 = padding row.
 #include "../lf_internal.cuh"
 
+#include <algorithm>
+#include <cstdio>
+#include <vector>
+
 namespace lf {
 
 namespace {
 
 constexpr unsigned kFull = 0xffffffffu;
 constexpr int kWarpsPerBlock = 8;
-constexpr int kChunk = 8;  // consecutive tasks per warp per round
+#ifndef LF_EPI_ZERO
+#define LF_EPI_ZERO 1  // empty C rows zeroed in the SpMM kernel's epilogue
+#endif
+constexpr int kChunk = kWideChunk;  // consecutive tasks per warp per round
 #ifndef LF_SPMM_MIN_BLOCKS
 #define LF_SPMM_MIN_BLOCKS 4
 #endif
@@ -99,6 +106,12 @@ template <> struct Vec<1> {
 __device__ __forceinline__ bool tag_whole(int32_t tag) { return (tag & 7) == 7; }  // S && F && L
 __device__ __forceinline__ int32_t tag_row(int32_t tag) { return tag >> 3; }
 
+#ifdef LF_TRACE
+__device__ unsigned long long lf_trace_buf[2 * 148 * 64];
+__device__ unsigned long long lf_trace_st[148 * 64];
+__device__ unsigned int lf_trace_tasks[148 * 64];
+__device__ unsigned long long lf_trace_t0;
+#endif
 // all-zero row that padding slots (colInd = -1, val = +0.0) gather from, so
 // every slot issues the same unpredicated load (JT <= 512 floats)
 __device__ float4 g_zero_row[128];
@@ -107,7 +120,10 @@ template <int VEC, int G, int NV>
 struct Layout {
     static constexpr int LPR = 32 / G;  // lanes per group
     static constexpr int JT = LPR * NV * VEC;
-    static constexpr int U = (8 / NV) > 1 ? (8 / NV) : 2;  // slots in flight per lane
+#ifndef LF_U
+#define LF_U 4
+#endif
+    static constexpr int U = (LF_U / NV) > 1 ? (LF_U / NV) : 2;  // slots in flight per lane
 };
 
 template <int VEC, int G, int NV, bool FULL>
@@ -206,9 +222,12 @@ __device__ __forceinline__ void fetch(const Cx &cx, const Resolved &r, int kb, t
     }
 }
 
-// the staged 32 slots accumulated into acc, no row boundary
+// the staged 32 slots accumulated into acc, no row boundary; slots at and
+// beyond n_real (a warp-uniform count: padding is a suffix of a CELL row)
+// are skipped a batch at a time
 template <class Cx>
-__device__ __forceinline__ void accum32(const Cx &cx, const Resolved &sw, typename Cx::VT (&acc)[Cx::NVv]) {
+__device__ __forceinline__ void accum32(const Cx &cx, const Resolved &sw, typename Cx::VT (&acc)[Cx::NVv],
+                                        int n_real = 32) {
     using V = typename Cx::V;
     using VT = typename Cx::VT;
     constexpr int NV = Cx::NVv;
@@ -216,6 +235,7 @@ __device__ __forceinline__ void accum32(const Cx &cx, const Resolved &sw, typena
     constexpr int U = Cx::L::U < STEPS ? Cx::L::U : STEPS;
 #pragma unroll
     for (int kb = 0; kb < STEPS; kb += U) {
+        if (kb * Cx::Gv >= n_real) break;
         VT b[U][NV];
         float a[U];
         fetch<Cx, U>(cx, sw, kb, b, a);
@@ -264,6 +284,30 @@ __device__ __forceinline__ void narrow_task(const Cx &cx, const Resolved &sw, in
     }
 }
 
+// Zero the C rows whose mode is in mode_mask (bit per kRow* value): the
+// rows that receive red.global.add must hold +0.0 first.  A warp scans 32 rows.
+__device__ __forceinline__ void zero_row(float *row, int J, int lane, bool vec4, uint64_t pol) {
+    if (vec4) {
+        for (int j = lane * 4; j < J; j += 128) Vec<4>::store(row + j, make_float4(0.f, 0.f, 0.f, 0.f), pol);
+    } else {
+        for (int j = lane; j < J; j += 32) row[j] = 0.f;
+    }
+}
+
+__device__ __forceinline__ void zero_rows_warp(const uint8_t *__restrict__ row_mode, int64_t n_rows, float *C,
+                                               int64_t ldc, int J, bool vec4, unsigned mode_mask, int64_t wid,
+                                               int64_t nw, int lane, uint64_t pol) {
+    for (int64_t base = wid * 32; base < n_rows; base += nw * 32) {
+        const int64_t i = base + lane;
+        unsigned need = __ballot_sync(kFull, i < n_rows && ((mode_mask >> __ldg(row_mode + i)) & 1u));
+        while (need) {
+            const int src = __ffs(need) - 1;
+            need &= need - 1;
+            zero_row(C + (base + src) * ldc, J, lane, vec4, pol);
+        }
+    }
+}
+
 // ---- asynchronous staging ----------------------------------------------
 // A warp owns two stage buffers; while it gathers B rows for the slots in
 // one, cp.async (LDGSTS, L2 evict_first) fills the other with the next
@@ -284,17 +328,22 @@ __device__ __forceinline__ void cp_async4(void *dst, const void *src, uint64_t p
 __device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void cp_wait1() { asm volatile("cp.async.wait_group 1;" ::: "memory"); }
 
-// chunked grid-stride task order: warp w takes tasks [w*CH, w*CH+CH), then
-// advances by nwarps*CH; returns the next task and flags the chunk end
-__device__ __forceinline__ int64_t next_task(int64_t task, int64_t &cs, int64_t round, int64_t n, bool &chunk_end) {
-    int64_t tn = task + 1;
-    chunk_end = false;
-    if (tn >= cs + kChunk || tn >= n) {
-        chunk_end = true;
-        cs += round;
-        tn = cs;
-    }
-    return tn;
+// ---- dynamic work queues --------------------------------------------------
+// Warps claim ranges of tasks with atomicAdd on per-launch counters (ctr[0]:
+// wide class, ctr[1]: narrow class).  Guided sizes: kChunk tasks while much
+// work remains, shrinking to 1 near the end so the last claims are short.  A
+// claim is issued one range ahead and read (shuffle from lane 0) only when
+// the warp moves on, so the atomic's latency is hidden; claims grow per warp,
+// so bucket cursors only move forward.
+__device__ __forceinline__ int claim_size(int64_t n, int64_t hint, int64_t nw) {
+    const int64_t left = n - hint;
+    return (int)max((int64_t)1, min((int64_t)kChunk, left / (2 * nw)));
+}
+__device__ __forceinline__ unsigned long long claim_issue(unsigned long long *ctr, int size, int lane) {
+    return lane == 0 ? atomicAdd(ctr, (unsigned long long)size) : 0ull;
+}
+__device__ __forceinline__ int64_t claim_get(unsigned long long raw) {
+    return (int64_t)__shfl_sync(kFull, raw, 0);
 }
 
 // W < 32 class: a task is 32 slots = 32/W rows of one bucket.  Returns t.
@@ -322,21 +371,29 @@ __device__ __forceinline__ int issue_narrow(const SpmmArgs &a, int64_t task, int
 }
 
 template <class Cx>
-__device__ __forceinline__ void narrow_loop(const SpmmArgs &a, const Cx &cx0, WarpStage &st, int lane, int64_t wid,
-                                            int64_t nw, uint64_t pol) {
+__device__ __forceinline__ void narrow_loop(const SpmmArgs &a, const Cx &cx0, WarpStage &st, int lane, int64_t nw,
+                                            uint64_t pol) {
     constexpr int G = Cx::Gv, JT = Cx::L::JT;
     Cx cx = cx0;
-    const int64_t round = nw * kChunk;
-    int64_t cs = wid * kChunk;
-    if (cs >= a.n_tasks_n) return;
+    const int64_t n = a.n_tasks_n;
+    int sz = claim_size(n, 0, nw);
+    int64_t task = claim_get(claim_issue(a.ctr + 1, sz, lane));
+    if (task >= n) return;
+    int64_t tend = min(task + sz, n);
+    int sz2 = claim_size(n, task, nw);
+    unsigned long long raw = claim_issue(a.ctr + 1, sz2, lane);
     int bcur = 0, buf = 0;
-    int64_t task = cs;
     int t = issue_narrow<G>(a, task, bcur, lane, pol, st, 0);
-    while (task < a.n_tasks_n) {
-        bool chunk_end;
-        const int64_t tn = next_task(task, cs, round, a.n_tasks_n, chunk_end);
+    while (task < n) {
+        int64_t tn = task + 1;
+        if (tn >= tend) {
+            tn = min(claim_get(raw), n);
+            tend = min(tn + sz2, n);
+            sz2 = claim_size(n, tn, nw);
+            raw = claim_issue(a.ctr + 1, sz2, lane);
+        }
         int tnext = 0;
-        if (tn < a.n_tasks_n) tnext = issue_narrow<G>(a, tn, bcur, lane, pol, st, buf ^ 1);
+        if (tn < n) tnext = issue_narrow<G>(a, tn, bcur, lane, pol, st, buf ^ 1);
         else cp_commit();
         cp_wait1();
         __syncwarp();
@@ -365,8 +422,8 @@ __device__ __forceinline__ void narrow_loop(const SpmmArgs &a, const Cx &cx0, Wa
 // W >= 32 class: a task is one CELL row = W/32 chunks of 32 slots.
 struct WideCursor {
     int64_t task;
-    int k, nch;       // chunk within the row, chunks per row
-    int last;         // task is the last of its warp chunk (flush pending runs after it)
+    int k, nch;  // 32-slot piece within the row, pieces per row
+    int last;    // task is the last of its warp chunk (flush pending runs after it)
 };
 
 template <int G>
@@ -387,37 +444,80 @@ __device__ __forceinline__ int wide_nch(const SpmmArgs &a, int64_t task, int &bc
     return 1 << (__ldg(&a.bk_w[bcur].t) - 5);
 }
 
+// Run-aligned claims: a claimed range [x, x + size) of the wide class really
+// covers [bound(x), bound(x + size)) with bound(x) = x + run_bound[x]
+// (run_bounds_kernel), so a whole run -- all CELL rows of a folded source
+// row, <= kMaxRun -- never straddles two warps and is one plain store.
+__device__ __forceinline__ int64_t chunk_bound(const SpmmArgs &a, int64_t x) {
+    return x >= a.n_tasks_w ? a.n_tasks_w : min(a.n_tasks_w, x + (int64_t)__ldg(a.run_bound + x));
+}
+
 template <class Cx>
-__device__ __forceinline__ void wide_loop(const SpmmArgs &a, const Cx &cx, WarpStage &st, int lane, int64_t wid,
-                                          int64_t nw, uint64_t pol) {
+__device__ __forceinline__ void wide_loop(const SpmmArgs &a, const Cx &cx, WarpStage &st, int lane, int64_t nw,
+                                          uint64_t pol) {
     using VT = typename Cx::VT;
     constexpr int NV = Cx::NVv, G = Cx::Gv;
-    const int64_t round = nw * kChunk;
-    int64_t cs = wid * kChunk;
-    if (cs >= a.n_tasks_w) return;
+    const int64_t n = a.n_tasks_w;
+    // current range [rs, re); next claimed range (x1, sz1) with its bounds
+    // loaded one range ahead; the claim after it in flight (raw, sz2)
+    int sz0 = claim_size(n, 0, nw);
+    int64_t x0 = claim_get(claim_issue(a.ctr, sz0, lane));
+    if (x0 >= n) return;
+    int sz1 = claim_size(n, x0, nw);
+    int64_t x1 = claim_get(claim_issue(a.ctr, sz1, lane));
+    int sz2 = claim_size(n, x1, nw);
+    unsigned long long raw = claim_issue(a.ctr, sz2, lane);
+    int64_t rs = chunk_bound(a, x0), re = chunk_bound(a, x0 + sz0);
+    int64_t nrs = chunk_bound(a, x1), nre = chunk_bound(a, x1 + sz1);
+    while (rs >= re && x0 < n) {  // empty range: its tasks belong to the previous range's run
+        x0 = x1;
+        rs = nrs;
+        re = nre;
+        x1 = claim_get(raw);
+        sz1 = sz2;
+        sz2 = claim_size(n, x1, nw);
+        raw = claim_issue(a.ctr, sz2, lane);
+        nrs = chunk_bound(a, x1);
+        nre = chunk_bound(a, x1 + sz1);
+    }
+    if (x0 >= n) return;
     int bcur = 0, buf = 0;
-    WideCursor cur{cs, 0, 0, 0};
+    WideCursor cur{rs, 0, 0, 0};
     cur.nch = wide_nch(a, cur.task, bcur);
     int bcur_cur = bcur;
     issue_wide<G>(a, cur, bcur, lane, pol, st, 0);
     VT acc[NV];
     cx.zero(acc);
-    int32_t pend = -1;      // tag of the run accumulated in acc (-1: none)
-    int32_t row_tag = -1;   // tag of the row being streamed
+    int32_t pend = -1;     // tag of the run accumulated in acc (-1: none)
+    int32_t row_tag = -1;  // tag of the row being streamed
     bool run_first = false;
-    while (cur.task < a.n_tasks_w) {
-        // successor chunk
+    while (cur.task < n) {
+        // successor piece: next 32 slots of the row, next task, or the first
+        // task of the warp's next non-empty chunk
         WideCursor nx = cur;
         if (cur.k + 1 < cur.nch) {
             nx.k = cur.k + 1;
         } else {
-            bool ce;
-            nx.task = next_task(cur.task, cs, round, a.n_tasks_w, ce);
             nx.k = 0;
-            cur.last = ce;
+            nx.task = cur.task + 1;
+            if (nx.task >= re) {
+                cur.last = 1;
+                do {
+                    x0 = x1;
+                    rs = nrs;
+                    re = nre;
+                    x1 = claim_get(raw);
+                    sz1 = sz2;
+                    sz2 = claim_size(n, x1, nw);
+                    raw = claim_issue(a.ctr, sz2, lane);
+                    nrs = chunk_bound(a, x1);
+                    nre = chunk_bound(a, x1 + sz1);
+                } while (rs >= re && x0 < n);
+                nx.task = x0 < n ? rs : n;
+            }
         }
         int bcur_nx = bcur_cur;
-        if (nx.task < a.n_tasks_w) {
+        if (nx.task < n) {
             if (nx.k == 0) {
                 nx.nch = wide_nch(a, nx.task, bcur);
                 bcur_nx = bcur;
@@ -440,11 +540,15 @@ __device__ __forceinline__ void wide_loop(const SpmmArgs &a, const Cx &cx, WarpS
                 if (pend < 0) run_first = (row_tag & 2) != 0;
             }
         }
-        if (row_tag >= 0 && __ballot_sync(kFull, st.slot[buf][lane].x >= 0)) {
+        const int n_real = row_tag >= 0 ? __popc(__ballot_sync(kFull, st.slot[buf][stage_pos<G>(lane)].x >= 0)) : 0;
+        if (n_real > 0) {
             resolve(cx, st.slot[buf], st.res, lane);
-            accum32(cx, st.res, acc);
+            accum32(cx, st.res, acc, n_real);
         }
         if (cur.k == cur.nch - 1) {
+#ifdef LF_TRACE
+            if (lane == 0) lf_trace_tasks[blockIdx.x * kWarpsPerBlock + (threadIdx.x >> 5)]++;
+#endif
             if (row_tag >= 0) {
                 pend = row_tag;
                 if (row_tag & 1) {  // last sub-row of the segment completes the run
@@ -472,56 +576,83 @@ __device__ __forceinline__ void wide_loop(const SpmmArgs &a, const Cx &cx, WarpS
 // synchronously, and every tile writes its slice (no run merging).
 template <class Cx>
 __device__ __forceinline__ void wide_loop_tiled(const SpmmArgs &a, const Cx &cx0, WarpStage &st, int lane,
-                                                int64_t wid, int64_t nw, uint64_t pol) {
+                                                uint64_t pol) {
     using VT = typename Cx::VT;
     constexpr int NV = Cx::NVv, G = Cx::Gv, JT = Cx::L::JT;
     Cx cx = cx0;
     int bcur = 0;
-    for (int64_t task = wid; task < a.n_tasks_w; task += nw) {
-        const int nch = wide_nch(a, task, bcur);
-        const BucketDev *bk = a.bk_w + bcur;
-        const int64_t tin = task - __ldg(&bk->task_off);
-        const int32_t tag = __ldg(a.row_tag + __ldg(&bk->row_off) + tin);
-        if (tag < 0) continue;
-        const int64_t s0 = __ldg(&bk->slot_off) + (tin << __ldg(&bk->t));
-        for (int j0 = 0; j0 < a.J; j0 += JT) {
-            cx.j0 = j0;
-            VT acc[NV];
-            cx.zero(acc);
-            for (int k = 0; k < nch; k++) {
-                const int32_t c_l = ld_stream(a.col + s0 + 32 * k + lane, pol);
-                const float v_l = ld_stream(a.val + s0 + 32 * k + lane, pol);
-                if (__ballot_sync(kFull, c_l >= 0) == 0) break;  // rest is padding
-                stage<G>(cx, st.res, lane, c_l, v_l);
-                accum32(cx, st.res, acc);
+    for (int64_t c = claim_get(claim_issue(a.ctr, kChunk, lane)); c < a.n_tasks_w;
+         c = claim_get(claim_issue(a.ctr, kChunk, lane))) {
+        for (int64_t task = c; task < min(c + kChunk, a.n_tasks_w); task++) {
+            const int nch = wide_nch(a, task, bcur);
+            const BucketDev *bk = a.bk_w + bcur;
+            const int64_t tin = task - __ldg(&bk->task_off);
+            const int32_t tag = __ldg(a.row_tag + __ldg(&bk->row_off) + tin);
+            if (tag < 0) continue;
+            const int64_t s0 = __ldg(&bk->slot_off) + (tin << __ldg(&bk->t));
+            for (int j0 = 0; j0 < a.J; j0 += JT) {
+                cx.j0 = j0;
+                VT acc[NV];
+                cx.zero(acc);
+                for (int k = 0; k < nch; k++) {
+                    const int32_t c_l = ld_stream(a.col + s0 + 32 * k + lane, pol);
+                    const float v_l = ld_stream(a.val + s0 + 32 * k + lane, pol);
+                    if (__ballot_sync(kFull, c_l >= 0) == 0) break;  // rest is padding
+                    stage<G>(cx, st.res, lane, c_l, v_l);
+                    accum32(cx, st.res, acc);
+                }
+                cx.reduce_groups(acc);
+                if (cx.g == 0) cx.write(tag_row(tag), tag_whole(tag), acc);
             }
-            cx.reduce_groups(acc);
-            if (cx.g == 0) cx.write(tag_row(tag), tag_whole(tag), acc);
         }
     }
 }
 
-// Blocks [0, a.blocks_n) run the W < 32 tasks, the rest the W >= 32 tasks:
-// the loops share no live state, so each is register-allocated alone.
+// Blocks [0, a.blocks_n) start on the W < 32 queue, the others on the
+// W >= 32 queue; a warp whose queue is drained helps with the other one.
+// The two loops run one after the other (no live state in common), so each
+// is register-allocated alone.  Epilogue: empty C rows are zeroed.
 template <int VEC, int G, int NV, bool FULL>
 __global__ void __launch_bounds__(kWarpsPerBlock * 32, kMinBlocks) cell_spmm_kernel(const SpmmArgs a) {
     using Cx = Ctx<VEC, G, NV, FULL>;
     using L = Layout<VEC, G, NV>;
     __shared__ __align__(16) WarpStage stage_buf[kWarpsPerBlock];
     const int lane = threadIdx.x & 31;
-    WarpStage &st = stage_buf[threadIdx.x >> 5];
+    const int w = threadIdx.x >> 5;
+    WarpStage &st = stage_buf[w];
     const uint64_t pol = policy_evict_first();
     const Cx cx{a.B, a.ldb, a.C, a.ldc, a.J, 0, lane / L::LPR, lane % L::LPR, pol};
-    const int w = threadIdx.x >> 5;
-    if ((int)blockIdx.x < a.blocks_n) {
-        narrow_loop(a, cx, st, lane, (int64_t)blockIdx.x * kWarpsPerBlock + w, (int64_t)a.blocks_n * kWarpsPerBlock,
-                    pol);
-    } else {
-        const int64_t wid = (int64_t)(blockIdx.x - a.blocks_n) * kWarpsPerBlock + w;
-        const int64_t nw = (int64_t)(gridDim.x - a.blocks_n) * kWarpsPerBlock;
-        if (a.J <= L::JT) wide_loop(a, cx, st, lane, wid, nw, pol);
-        else wide_loop_tiled(a, cx, st, lane, wid, nw, pol);
+    const bool tiled = a.J > L::JT;
+#ifdef LF_TRACE
+    {
+        unsigned long long t0;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+        if (lane == 0) { lf_trace_st[blockIdx.x * kWarpsPerBlock + w] = t0; lf_trace_tasks[blockIdx.x * kWarpsPerBlock + w] = 0; }
     }
+#endif
+    const int64_t nw = (int64_t)gridDim.x * kWarpsPerBlock;
+    if ((int)blockIdx.x < a.blocks_n) {
+        narrow_loop(a, cx, st, lane, nw, pol);
+        if (tiled) wide_loop_tiled(a, cx, st, lane, pol);
+        else wide_loop(a, cx, st, lane, nw, pol);
+    } else {
+        if (tiled) wide_loop_tiled(a, cx, st, lane, pol);
+        else wide_loop(a, cx, st, lane, nw, pol);
+        narrow_loop(a, cx, st, lane, nw, pol);
+    }
+#ifdef LF_TRACE
+    unsigned long long t_work;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_work));
+#endif
+    if (LF_EPI_ZERO)
+        zero_rows_warp(a.row_mode, a.n_rows, a.C, a.ldc, a.J, VEC == 4, 1u << kRowEmpty,
+                       (int64_t)blockIdx.x * kWarpsPerBlock + w, (int64_t)gridDim.x * kWarpsPerBlock, lane, pol);
+#ifdef LF_TRACE
+    if (lane == 0) lf_trace_buf[(blockIdx.x * kWarpsPerBlock + w) * 2] = t_work;
+    unsigned long long t_end;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_end));
+    if (lane == 0) lf_trace_buf[(blockIdx.x * kWarpsPerBlock + w) * 2 + 1] = t_end;
+#endif
 }
 
 // Algorithm 1 on the GPU straight from CSR: one warp per row, same lane layout.
@@ -558,28 +689,13 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32)
     }
 }
 
-// C rows whose source row has != 1 CELL rows: zero (empty rows are the
-// result; multi-writer rows then receive red.add).  A warp scans 32 rows.
-__global__ void zero_rows_kernel(const int32_t *__restrict__ row_cnt, int64_t n_rows, float *__restrict__ C,
-                                 int64_t ldc, int J, int vec4) {
+__global__ void zero_rows_kernel(const uint8_t *__restrict__ row_mode, int64_t n_rows, float *__restrict__ C,
+                                 int64_t ldc, int J, int vec4, unsigned mode_mask) {
     const int lane = threadIdx.x & 31;
     const int64_t gwarp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    for (int64_t base = gwarp * 32; base < n_rows; base += nwarps * 32) {
-        const int64_t i = base + lane;
-        unsigned need = __ballot_sync(kFull, i < n_rows && __ldg(row_cnt + i) != 1);
-        while (need) {
-            const int src = __ffs(need) - 1;
-            need &= need - 1;
-            float *row = C + (base + src) * ldc;
-            if (vec4) {
-                for (int j = lane * 4; j < J; j += 128)
-                    *reinterpret_cast<float4 *>(row + j) = make_float4(0.f, 0.f, 0.f, 0.f);
-            } else {
-                for (int j = lane; j < J; j += 32) row[j] = 0.f;
-            }
-        }
-    }
+    zero_rows_warp(row_mode, n_rows, C, ldc, J, vec4 != 0, mode_mask, gwarp, nwarps, lane,
+                   policy_evict_first());
 }
 
 template <typename F>
@@ -607,10 +723,53 @@ cudaError_t run_cell(const SpmmArgs &a0, cudaStream_t s) {
     bn = std::min(bn, want_n);
     bw = std::min(bw, want_w);
     a.blocks_n = (int)bn;
-    const int grid = (int)(bn + bw);
+    // enough blocks for the empty-row epilogue even without tasks
+    const int64_t want_z = std::min<int64_t>(cap, (a.n_rows + 32 * kWarpsPerBlock - 1) / (32 * kWarpsPerBlock));
+    const int grid = (int)std::max<int64_t>(bn + bw, want_z);
     if (grid == 0) return cudaSuccess;
+    // per-launch queue counters (stream-ordered), so concurrent calls on one
+    // handle stay independent
+    unsigned long long *ctr = nullptr;
+    cudaError_t e = cudaMallocAsync(&ctr, 2 * sizeof(unsigned long long), s);
+    if (e != cudaSuccess) return e;
+    if ((e = cudaMemsetAsync(ctr, 0, 2 * sizeof(unsigned long long), s)) != cudaSuccess) return e;
+    a.ctr = ctr;
     fn<<<grid, kWarpsPerBlock * 32, 0, s>>>(a);
-    return cudaGetLastError();
+    if ((e = cudaGetLastError()) != cudaSuccess) return e;
+#ifdef LF_TRACE
+    {
+        static std::vector<unsigned long long> h(2 * 148 * 64);
+        cudaStreamSynchronize(s);
+        cudaMemcpyFromSymbol(h.data(), lf_trace_buf, h.size() * 8);
+        static std::vector<unsigned long long> hs(148 * 64);
+        static std::vector<unsigned int> ht(148 * 64);
+        cudaMemcpyFromSymbol(hs.data(), lf_trace_st, hs.size() * 8);
+        cudaMemcpyFromSymbol(ht.data(), lf_trace_tasks, ht.size() * 4);
+        const int nw = grid * kWarpsPerBlock;
+        unsigned long long mn = ~0ull, mx = 0;
+        for (int i = 0; i < nw; i++) { mn = std::min(mn, hs[i]); mx = std::max(mx, h[2 * i + 1]); }
+        {
+            std::vector<unsigned> tt(ht.begin() + a.blocks_n * kWarpsPerBlock, ht.begin() + nw);
+            std::sort(tt.begin(), tt.end());
+            std::vector<double> st0;
+            for (int i = 0; i < nw; i++) st0.push_back((hs[i] - mn) / 1e3);
+            std::sort(st0.begin(), st0.end());
+            fprintf(stderr, "trace: wide-block warps tasks p0 %u p50 %u p99 %u max %u | start us p50 %.1f max %.1f\n", tt[0], tt[tt.size() / 2],
+                    tt[tt.size() * 99 / 100], tt.back(), st0[nw / 2], st0[nw - 1]);
+            // slowest warp
+            int sl = 0;
+            for (int i = 0; i < nw; i++) if (h[2 * i] > h[2 * sl]) sl = i;
+            fprintf(stderr, "trace: slowest warp %d (block %d) tasks %u work_end %.1f\n", sl, sl / kWarpsPerBlock, ht[sl], (h[2 * sl] - mn) / 1e3);
+        }
+        std::vector<double> wk, en;
+        for (int i = 0; i < nw; i++) { wk.push_back((h[2 * i] - mn) / 1e3); en.push_back((h[2 * i + 1] - mn) / 1e3); }
+        std::sort(wk.begin(), wk.end());
+        std::sort(en.begin(), en.end());
+        fprintf(stderr, "trace: warps=%d blocks_n=%d work_end us: p0 %.1f p10 %.1f p50 %.1f p90 %.1f p100 %.1f | epi end p50 %.1f p100 %.1f\n",
+                nw, a.blocks_n, wk[0], wk[nw / 10], wk[nw / 2], wk[nw * 9 / 10], wk[nw - 1], en[nw / 2], en[nw - 1]);
+    }
+#endif
+    return cudaFreeAsync(ctr, s);
 }
 
 template <int VEC, int G, int NV>
@@ -641,18 +800,25 @@ bool vec4_ok(const float *B, int64_t ldb, const float *C, int64_t ldc, int J) {
 
 }  // namespace
 
-cudaError_t launch_zero_rows(const int32_t *row_cnt, int64_t n_rows, float *C, int64_t ldc, int J, cudaStream_t s) {
-    if (n_rows == 0 || J == 0) return cudaSuccess;
-    const int vec4 = (J % 4 == 0 && ldc % 4 == 0 && ((uintptr_t)C & 15) == 0) ? 1 : 0;
-    int64_t warps = (n_rows + 31) / 32;
+// rows written with red.global.add must be zero first: kRowRed always, and
+// kRowRun rows too when J needs several tiles (no run merging then)
+cudaError_t zero_red_rows(const SpmmArgs &a, bool tiled, cudaStream_t s) {
+    if (a.n_rows == 0 || a.J == 0) return cudaSuccess;
+    const int vec4 = (a.J % 4 == 0 && a.ldc % 4 == 0 && ((uintptr_t)a.C & 15) == 0) ? 1 : 0;
+    const unsigned mask = (1u << kRowRed) | (tiled ? (1u << kRowRun) : 0u) | (LF_EPI_ZERO ? 0u : (1u << kRowEmpty));
+    int64_t warps = (a.n_rows + 31) / 32;
     int grid = (int)std::max<int64_t>(1, std::min<int64_t>((warps + 7) / 8, 148LL * 16));
-    zero_rows_kernel<<<grid, 256, 0, s>>>(row_cnt, n_rows, C, ldc, J, vec4);
+    zero_rows_kernel<<<grid, 256, 0, s>>>(a.row_mode, a.n_rows, a.C, a.ldc, a.J, vec4, mask);
     return cudaGetLastError();
 }
 
 cudaError_t launch_cell_spmm(const SpmmArgs &a, cudaStream_t s) {
-    if (a.n_tasks_n + a.n_tasks_w == 0 || a.J == 0) return cudaSuccess;
-    if (vec4_ok(a.B, a.ldb, a.C, a.ldc, a.J)) {
+    if (a.J == 0 || a.n_rows == 0) return cudaSuccess;
+    const bool v4 = vec4_ok(a.B, a.ldb, a.C, a.ldc, a.J);
+    const bool tiled = v4 ? a.J > 512 : a.J > 128;
+    cudaError_t e = zero_red_rows(a, tiled, s);
+    if (e != cudaSuccess) return e;
+    if (v4) {
         if (a.J <= 32) return run_cell_j<4, 4, 1>(a, s);
         if (a.J <= 64) return run_cell_j<4, 2, 1>(a, s);
         if (a.J <= 128) return run_cell_j<4, 1, 1>(a, s);

@@ -283,8 +283,10 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
     bs.tile_cnt = sc.get<long long>((size_t)P * lf::kMaxT * std::max(n_tiles, 1));
     bs.key_total = sc.get<long long>((size_t)P * lf::kMaxT);
     bs.key_row_off = sc.get<long long>((size_t)P * lf::kMaxT);
-    h->row_cnt = static_cast<int32_t *>(mem.get((size_t)std::max<int64_t>(I, 1) * sizeof(int32_t)));
-    if (!d_e || !bs.tile_cnt || !bs.key_total || !bs.key_row_off || !h->row_cnt || (P > 1 && I > 0 && !bs.seg_rel))
+    int32_t *row_cnt = sc.get<int32_t>((size_t)std::max<int64_t>(I, 1));
+    h->row_mode = static_cast<uint8_t *>(mem.get((size_t)std::max<int64_t>(I, 1)));
+    if (!d_e || !bs.tile_cnt || !bs.key_total || !bs.key_row_off || !row_cnt || !h->row_mode ||
+        (P > 1 && I > 0 && !bs.seg_rel))
         return bail(fail(LF_ERR_NO_MEMORY, "scratch allocation failed"));
 
     // a1 + a4 (count): segments, bucket keys, per-tile totals, tile scan
@@ -295,12 +297,14 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
     lf_status st;
     if ((st = cu(cudaMemcpyAsync(d_e, params->max_width_log2, LF_MAX_PARTS, cudaMemcpyHostToDevice, s), "H2D e")))
         return bail(st);
-    if ((st = cu(cudaMemsetAsync(h->row_cnt, 0, (size_t)std::max<int64_t>(I, 1) * sizeof(int32_t), s), "memset")))
+    if ((st = cu(cudaMemsetAsync(row_cnt, 0, (size_t)std::max<int64_t>(I, 1) * sizeof(int32_t), s), "memset")))
+        return bail(st);
+    if ((st = cu(cudaMemsetAsync(h->row_mode, lf::kRowEmpty, (size_t)std::max<int64_t>(I, 1), s), "memset")))
         return bail(st);
     if ((st = cu(cudaMemsetAsync(bs.tile_cnt, 0, (size_t)P * lf::kMaxT * std::max(n_tiles, 1) * 8, s), "memset")))
         return bail(st);
     if ((st = cu(lf::launch_seg(*A, P, bs.seg_rel, s), "seg"))) return bail(st);
-    if ((st = cu(lf::launch_bucket_count(*A, P, d_e, bs, h->row_cnt, s), "bucket_count"))) return bail(st);
+    if ((st = cu(lf::launch_bucket_count(*A, P, d_e, bs, row_cnt, s), "bucket_count"))) return bail(st);
     if (n_tiles > 0 && (st = cu(lf::launch_tile_scan(P, bs, s), "tile_scan"))) return bail(st);
     std::vector<long long> tot((size_t)P * lf::kMaxT, 0);
     if (n_tiles > 0 &&
@@ -365,8 +369,9 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
     const size_t a256 = 256;
     auto up = [&](size_t b) { return (b + a256 - 1) / a256 * a256; };
     const size_t b_ri = up(R_tot * 4), b_rt = up(R_tot * 4), b_ci = up(S_tot * 4), b_va = up(S_tot * 4),
-                 b_bk = up(h->h_buckets.size() * sizeof(lf::BucketDev));
-    h->pool_bytes = b_ri + b_rt + b_ci + b_va + b_bk;
+                 b_bk = up(h->h_buckets.size() * sizeof(lf::BucketDev)),
+                 b_rb = up((size_t)(h->n_tasks_w + 1));
+    h->pool_bytes = b_ri + b_rt + b_ci + b_va + b_bk + b_rb;
     h->pool = mem.get(h->pool_bytes);
     if (h->pool_bytes && !h->pool) return bail(fail(LF_ERR_NO_MEMORY, "CELL arrays allocation failed"));
     char *q = static_cast<char *>(h->pool);
@@ -375,6 +380,7 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
     h->col_ind = reinterpret_cast<int32_t *>(q + b_ri + b_rt);
     h->val = reinterpret_cast<float *>(q + b_ri + b_rt + b_ci);
     h->d_buckets = reinterpret_cast<lf::BucketDev *>(q + b_ri + b_rt + b_ci + b_va);
+    h->run_bound = reinterpret_cast<uint8_t *>(q + b_ri + b_rt + b_ci + b_va + b_bk);
     bs.src_pos = sc.get<int64_t>((size_t)R_tot);
     bs.src_cnt = sc.get<int32_t>((size_t)R_tot);
     if (R_tot && (!bs.src_pos || !bs.src_cnt)) return bail(fail(LF_ERR_NO_MEMORY, "scratch allocation failed"));
@@ -392,9 +398,15 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
                  "H2D row_off")))
         return bail(st);
     // a4 (place) + a5 (scatter)
-    if ((st = cu(lf::launch_bucket_place(*A, P, d_e, bs, h->row_cnt, h->row_ind, h->row_tag, s), "bucket_place")))
+    if ((st = cu(lf::launch_bucket_place(*A, P, d_e, bs, row_cnt, h->row_ind, h->row_tag, h->row_mode, s),
+                 "bucket_place")))
         return bail(st);
     if ((st = cu(lf::launch_slot_fill(*A, h->d_buckets, nb, S_tot, bs, h->col_ind, h->val, s), "slot_fill")))
+        return bail(st);
+    if (h->pool &&
+        (st = cu(lf::launch_run_bounds(h->d_buckets + nb + h->nb_n, h->nb_w, h->n_tasks_w, h->row_tag, h->run_bound,
+                                       s),
+                 "run_bounds")))
         return bail(st);
     *out = h;
     return LF_OK;
@@ -413,10 +425,11 @@ lf_status lf_spmm(const lf_cell *h, const float *B, int64_t ldb, int32_t J, floa
         LF_CUDA(lf::launch_csr_spmm(h->csr, B, ldb, J, C, ldc, s));
         return LF_OK;
     }
-    LF_CUDA(lf::launch_zero_rows(h->row_cnt, h->n_rows, C, ldc, J, s));
     const int nb = (int)h->buckets.size();
     lf::SpmmArgs a{h->d_buckets + nb, h->d_buckets + nb + h->nb_n, h->nb_n, h->nb_w, h->n_tasks_n, h->n_tasks_w,
-                   h->slots_n, h->slots_w, 0, h->col_ind, h->val, h->row_tag, B, ldb, C, ldc, J};
+                   h->slots_n, h->slots_w, 0, h->row_mode, h->n_rows, h->run_bound, nullptr, h->col_ind, h->val,
+                   h->row_tag,
+                   B, ldb, C, ldc, J};
     LF_CUDA(lf::launch_cell_spmm(a, s));
     return LF_OK;
 }
@@ -453,7 +466,7 @@ lf_status lf_cell_destroy(lf_cell *h) {
     if (!h) return LF_OK;
     Mem mem{h->custom_al ? &h->al : nullptr, h->stream};
     mem.put(h->pool, h->pool_bytes);
-    mem.put(h->row_cnt, (size_t)std::max<int64_t>(h->n_rows, 1) * sizeof(int32_t));
+    mem.put(h->row_mode, (size_t)std::max<int64_t>(h->n_rows, 1));
     delete h;
     return LF_OK;
 }

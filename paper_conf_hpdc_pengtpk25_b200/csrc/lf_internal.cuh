@@ -61,13 +61,36 @@ struct BuildScratch {
     int n_tiles;
 };
 constexpr int kBuildTile = 256;  // rows per tile of the bucketize passes
+// A folded source row whose CELL rows all sit in one wide bucket (W >= 32)
+// and number at most kMaxRun is summed by a single warp and stored once.
+#ifndef LF_MAX_RUN
+#define LF_MAX_RUN 8
+#endif
+constexpr int kMaxRun = LF_MAX_RUN;
+// Work is claimed from per-launch queues in ranges of at most kWideChunk
+// tasks (smaller near the end); run_bound[x] = offset (0..32) from wide task x
+// to the first task that may start a claim (never inside a whole run).
+#ifndef LF_WIDE_CHUNK
+#define LF_WIDE_CHUNK 8
+#endif
+constexpr int kWideChunk = LF_WIDE_CHUNK;
+// row_mode[i]: how C row i is produced
+enum : uint8_t {
+    kRowPlain = 0,  // one CELL row, plain store
+    kRowEmpty = 1,  // no CELL row: zeroed by the SpMM kernel's epilogue
+    kRowRed = 2,    // several writers: pre-zeroed, red.global.add
+    kRowRun = 3,    // a whole run (<= kMaxRun CELL rows) summed by one warp, plain store
+};
 
 cudaError_t launch_seg(const lf_csr &A, int P, int32_t *seg_rel, cudaStream_t s);
 cudaError_t launch_bucket_count(const lf_csr &A, int P, const int8_t *e, const BuildScratch &sc,
                                 int32_t *row_cnt, cudaStream_t s);
 cudaError_t launch_tile_scan(int P, const BuildScratch &sc, cudaStream_t s);
 cudaError_t launch_bucket_place(const lf_csr &A, int P, const int8_t *e, const BuildScratch &sc,
-                                const int32_t *row_cnt, int32_t *row_ind, int32_t *row_tag, cudaStream_t s);
+                                const int32_t *row_cnt, int32_t *row_ind, int32_t *row_tag, uint8_t *row_mode,
+                                cudaStream_t s);
+cudaError_t launch_run_bounds(const BucketDev *bk_w, int nb_w, int64_t n_tasks_w, const int32_t *row_tag,
+                              uint8_t *run_bound, cudaStream_t s);
 cudaError_t launch_slot_fill(const lf_csr &A, const BucketDev *d_buckets, int nb, int64_t n_slots,
                              const BuildScratch &sc, int32_t *col_out, float *val_out, cudaStream_t s);
 
@@ -79,6 +102,10 @@ struct SpmmArgs {
     int64_t n_tasks_n, n_tasks_w;
     int64_t slots_n, slots_w;
     int blocks_n;  // set by the launcher
+    const uint8_t *row_mode;
+    int64_t n_rows;
+    const uint8_t *run_bound;  // [n_tasks_w + 1]
+    unsigned long long *ctr;   // per-launch work-queue counters (set by the launcher)
     const int32_t *col;
     const float *val;
     const int32_t *row_tag;
@@ -88,8 +115,7 @@ struct SpmmArgs {
     int64_t ldc;
     int J;
 };
-cudaError_t launch_zero_rows(const int32_t *row_cnt, int64_t n_rows, float *C, int64_t ldc, int J, cudaStream_t s);
-cudaError_t launch_cell_spmm(const SpmmArgs &a, cudaStream_t s);
+cudaError_t launch_cell_spmm(const SpmmArgs &a, cudaStream_t s);  // pre-zeroes kRowRed rows itself
 cudaError_t launch_csr_spmm(const lf_csr &A, const float *B, int64_t ldb, int J, float *C, int64_t ldc,
                             cudaStream_t s);
 cudaError_t launch_validate(const lf_csr &A, int *d_flag, cudaStream_t s);
@@ -106,7 +132,8 @@ struct lf_cell {
     int32_t *col_ind = nullptr;
     float *val = nullptr;
     int32_t *row_tag = nullptr;  // (row << 3) | S,F,L flags (cell_spmm.cu); -1 = padding
-    int32_t *row_cnt = nullptr;  // CELL rows per source row
+    uint8_t *row_mode = nullptr;  // [n_rows] kRow* (how each C row is produced)
+    uint8_t *run_bound = nullptr; // [n_tasks_w + 1] (in the pool)
     lf::BucketDev *d_buckets = nullptr;  // [nb] all, then [nb_n] W < 32 class, then [nb_w] W >= 32 class
     std::vector<lf_bucket> buckets;
     std::vector<lf::BucketDev> h_buckets;
