@@ -241,7 +241,7 @@ def main():
         e0 = ev(); e0.record(stream)
         params, stats = lf.configure(Ain, J, **kw)
         e1 = ev(); e1.record(stream)
-        M = lf.CellMatrix.build(Ain, params)
+        M = lf.CellMatrix.build(Ain, params, stats)
         e2 = ev(); e2.record(stream)
         M.spmm(d_B, out=C_loc)
         e3 = ev(); e3.record(stream)
@@ -295,8 +295,8 @@ def main():
     ph = {k: maxr(v) for k, v in ph.items()}
 
     # ---- SpMM alone (the paper's kernel-only time) -----------
-    params, _ = lf.configure(A, J, **kw)
-    M = lf.CellMatrix.build(A, params)
+    params, stats = lf.configure(A, J, **kw)
+    M = lf.CellMatrix.build(A, params, stats)
     for _ in range(3):
         M.spmm(d_B, out=C_loc)
     torch.cuda.synchronize()
@@ -319,8 +319,8 @@ def main():
             for hs, ds in ((h_rp, d_rp), (h_ci, d_ci), (h_va, d_va), (h_B, d_B)):
                 ds.copy_(hs, non_blocking=True)
             Ain = lf.Csr(d_rp, d_ci, d_va, A_h.n_cols, p1 - p0)
-            pr, _ = lf.configure(Ain, J, **kw)
-            Mi = lf.CellMatrix.build(Ain, pr)
+            pr, sti = lf.configure(Ain, J, **kw)
+            Mi = lf.CellMatrix.build(Ain, pr, sti)
             Mi.spmm(d_B, out=C_loc)
             if world > 1:
                 lfd.gather_rows(C_loc, bounds)

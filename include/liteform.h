@@ -197,14 +197,19 @@ LF_API lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configur
 
 /* CSR -> CELL conversion on the GPU (section 4; canonical layout R1-R7; the
  * output is bit-identical to the oracle's).  Allocates the handle's arrays
- * through al (NULL = cudaMallocAsync).  Synchronises s once (to learn the
- * bucket sizes); the rest is enqueued asynchronously on s, so the handle may
- * be used on s immediately.
- * Errors: LF_ERR_INVALID_ARG (sizes, e_p > k_p, P out of range),
- *         LF_ERR_INDEX_OVERFLOW (n_rows >= 2^28 or K > 2^31-1),
+ * through al (NULL = cudaMallocAsync).
+ *   stats   (host, may be NULL) the statistics lf_cell_configure returned for
+ *           the SAME A with params->n_parts partitions: the bucket sizes follow
+ *           from them (bucket t < e_p holds H[p][t] rows, the max bucket
+ *           F[p][e_p]), so the build enqueues everything asynchronously with
+ *           no host synchronisation.  NULL: the sizes are counted on the GPU
+ *           and s is synchronised once.
+ * The handle may be used on s immediately.
+ * Errors: LF_ERR_INVALID_ARG (sizes, e_p > k_p, P out of range, stats for a
+ *         different P), LF_ERR_INDEX_OVERFLOW (n_rows >= 2^28 or K > 2^31-1),
  *         LF_ERR_NO_MEMORY, LF_ERR_CUDA, LF_ERR_UNSORTED_CSR (LF_VALIDATE=1). */
-LF_API lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_allocator *al, lf_stream_t s,
-                        lf_cell **out);
+LF_API lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_configure_stats *stats,
+                               const lf_allocator *al, lf_stream_t s, lf_cell **out);
 
 /* C = A . B (eq. 3-4; Alg. 2 over every block),
  * overwriting C (beta = 0; rows of A with no entries become +0.0, R13).

@@ -115,11 +115,14 @@ class CellMatrix:
         self.n_cols = A.n_cols
 
     @staticmethod
-    def build(A: Csr, params: LfCellParams, stream=None) -> "CellMatrix":
+    def build(A: Csr, params: LfCellParams, stats: LfConfigureStats | None = None, stream=None) -> "CellMatrix":
+        """GPU CSR -> CELL.  Passing the stats lf.configure returned for this A
+        lets the build run without a host synchronisation."""
         h = ctypes.c_void_p()
         csr = A.c()
-        _abi.check(lib.lf_cell_build(ctypes.byref(csr), ctypes.byref(params), ctypes.byref(_abi.torch_allocator()),
-                                     _stream(stream), ctypes.byref(h)))
+        _abi.check(lib.lf_cell_build(ctypes.byref(csr), ctypes.byref(params),
+                                     ctypes.byref(stats) if stats is not None else None,
+                                     ctypes.byref(_abi.torch_allocator()), _stream(stream), ctypes.byref(h)))
         return CellMatrix(h, A, params)
 
     def spmm(self, B: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:

@@ -80,8 +80,8 @@ class LfCellArrays(ctypes.Structure):
 SIGNATURES = {
     "lf_cell_configure": (_I32, [ctypes.POINTER(LfCsr), _I32, ctypes.POINTER(LfConfigureOpts),
                                  ctypes.POINTER(LfCellParams), ctypes.POINTER(LfConfigureStats), _P]),
-    "lf_cell_build": (_I32, [ctypes.POINTER(LfCsr), ctypes.POINTER(LfCellParams), ctypes.POINTER(LfAllocator), _P,
-                             ctypes.POINTER(ctypes.c_void_p)]),
+    "lf_cell_build": (_I32, [ctypes.POINTER(LfCsr), ctypes.POINTER(LfCellParams), ctypes.POINTER(LfConfigureStats),
+                             ctypes.POINTER(LfAllocator), _P, ctypes.POINTER(ctypes.c_void_p)]),
     "lf_spmm": (_I32, [_P, _P, _I64, _I32, _P, _I64, _P]),
     "lf_csr_spmm": (_I32, [ctypes.POINTER(LfCsr), _P, _I64, _I32, _P, _I64, _P]),
     "lf_cell_view": (_I32, [_P, ctypes.POINTER(LfCellArrays)]),

@@ -122,8 +122,8 @@ __global__ void __launch_bounds__(kThreads) stats_rows_kernel(const int64_t *__r
     }
     __syncthreads();
     for (int q = threadIdx.x; q < P * kMaxT; q += blockDim.x) {
-        if (H_s[q]) atomicAdd(&st->H[0][0] + q, H_s[q]);
-        if (F_s[q]) atomicAdd(&st->F[0][0] + q, F_s[q]);
+        if (H_s[q]) atomicAdd(&st->part[q / kMaxT].H[q % kMaxT], H_s[q]);
+        if (F_s[q]) atomicAdd(&st->part[q / kMaxT].F[q % kMaxT], F_s[q]);
     }
 }
 
@@ -273,8 +273,8 @@ __global__ void __launch_bounds__(kThreads) stats_cols_kernel(const uint32_t *__
     }
     __syncthreads();
     for (int q = threadIdx.x; q < P * kMaxT; q += blockDim.x) {
-        if (Un_s[q]) atomicAdd(&st->Unat[0][0] + q, Un_s[q]);
-        if (Ut_s[q]) atomicAdd(&st->Utop[0][0] + q, Ut_s[q]);
+        if (Un_s[q]) atomicAdd(&st->part[q / kMaxT].Unat[q % kMaxT], Un_s[q]);
+        if (Ut_s[q]) atomicAdd(&st->part[q / kMaxT].Utop[q % kMaxT], Ut_s[q]);
     }
 }
 

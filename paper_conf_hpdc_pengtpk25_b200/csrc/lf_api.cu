@@ -164,8 +164,9 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
     const int P = o.force_parts ? o.force_parts : standin_parts(A, J, max_parts);
     lf::StatsDev *d_st = nullptr;
     uint32_t *d_mask = nullptr;
-    LF_CUDA(cudaMallocAsync(&d_st, sizeof(lf::StatsDev), s));
-    LF_CUDA(cudaMemsetAsync(d_st, 0, sizeof(lf::StatsDev), s));
+    const size_t st_bytes = lf::stats_bytes(P);
+    LF_CUDA(cudaMallocAsync(&d_st, st_bytes, s));
+    LF_CUDA(cudaMemsetAsync(d_st, 0, st_bytes, s));
     LF_CUDA(cudaMemsetAsync(&d_st->len_min, 0xFF, sizeof(unsigned long long), s));
     if (A->n_cols > 0) {
         const size_t words = lf::mask_slots(A->n_cols);
@@ -175,13 +176,15 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
     uint8_t *d_t0 = nullptr;
     if (A->n_rows > 0) LF_CUDA(cudaMallocAsync(&d_t0, lf::stats_scratch_bytes(A->n_rows, A->nnz, P), s));
     LF_CUDA(lf::launch_stats(*A, P, d_st, d_mask, d_t0, s));
-    std::vector<lf::StatsDev> h(1);
-    LF_CUDA(cudaMemcpyAsync(h.data(), d_st, sizeof(lf::StatsDev), cudaMemcpyDeviceToHost, s));
+    // pinned staging buffer (one per thread) so the copy back is a plain DMA
+    thread_local lf::StatsDev *h_st = nullptr;
+    if (!h_st) LF_CUDA(cudaMallocHost(&h_st, sizeof(lf::StatsDev)));
+    LF_CUDA(cudaMemcpyAsync(h_st, d_st, st_bytes, cudaMemcpyDeviceToHost, s));
     LF_CUDA(cudaFreeAsync(d_st, s));
     if (d_mask) LF_CUDA(cudaFreeAsync(d_mask, s));
     if (d_t0) LF_CUDA(cudaFreeAsync(d_t0, s));
     LF_CUDA(cudaStreamSynchronize(s));
-    const lf::StatsDev &st = h[0];
+    const lf::StatsDev &st = *h_st;
 
     lf_configure_stats local;
     lf_configure_stats &cs = stats ? *stats : local;
@@ -205,12 +208,12 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
     for (int p = 0; p < P; p++) {
         int top = -1;
         for (int t = 0; t < lf::kMaxT; t++) {
-            cs.H[p][t] = (int64_t)st.H[p][t];
-            cs.F[p][t] = (int64_t)st.F[p][t];
-            cs.Unat[p][t] = (int64_t)st.Unat[p][t];
-            cs.Utop[p][t] = (int64_t)st.Utop[p][t];
+            cs.H[p][t] = (int64_t)st.part[p].H[t];
+            cs.F[p][t] = (int64_t)st.part[p].F[t];
+            cs.Unat[p][t] = (int64_t)st.part[p].Unat[t];
+            cs.Utop[p][t] = (int64_t)st.part[p].Utop[t];
             cs.cost[p][t] = -1;
-            if (st.H[p][t]) top = t;
+            if (st.part[p].H[t]) top = t;
         }
         cs.max_log2[p] = top;
         // eq. 7 (reading R10): buckets b < e keep their natural rows,
@@ -234,8 +237,8 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
     return LF_OK;
 }
 
-lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_allocator *al, lf_stream_t stream,
-                        lf_cell **out) {
+lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_configure_stats *stats,
+                        const lf_allocator *al, lf_stream_t stream, lf_cell **out) {
     g_detail.clear();
     if (lf_status st = check_csr(A)) return st;
     if (!params || !out) return fail(LF_ERR_INVALID_ARG, "params/out is NULL");
@@ -249,6 +252,7 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
             return fail(LF_ERR_INVALID_ARG, "need 0 <= e_p <= k_p <= 30");
     }
     if (al && (!al->alloc || !al->free)) return fail(LF_ERR_INVALID_ARG, "allocator without alloc/free");
+    if (stats && stats->n_parts != P) return fail(LF_ERR_INVALID_ARG, "stats were computed for another n_parts");
     cudaStream_t s = (cudaStream_t)stream;
     if (lf_status st = maybe_validate(A, s)) return st;
     keep_default_pool();
@@ -307,10 +311,18 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
     if ((st = cu(lf::launch_bucket_count(*A, P, d_e, bs, row_cnt, s), "bucket_count"))) return bail(st);
     if (n_tiles > 0 && (st = cu(lf::launch_tile_scan(P, bs, s), "tile_scan"))) return bail(st);
     std::vector<long long> tot((size_t)P * lf::kMaxT, 0);
-    if (n_tiles > 0 &&
-        (st = cu(cudaMemcpyAsync(tot.data(), bs.key_total, tot.size() * 8, cudaMemcpyDeviceToHost, s), "D2H")))
-        return bail(st);
-    if ((st = cu(cudaStreamSynchronize(s), "sync"))) return bail(st);
+    if (stats) {  // bucket sizes from the configure statistics: no synchronisation
+        for (int p = 0; p < P; p++) {
+            const int e = params->max_width_log2[p];
+            for (int t = 0; t < e && t < lf::kMaxT; t++) tot[(size_t)p * lf::kMaxT + t] = stats->H[p][t];
+            if (e < lf::kMaxT) tot[(size_t)p * lf::kMaxT + e] = stats->F[p][e];
+        }
+    } else {
+        if (n_tiles > 0 &&
+            (st = cu(cudaMemcpyAsync(tot.data(), bs.key_total, tot.size() * 8, cudaMemcpyDeviceToHost, s), "D2H")))
+            return bail(st);
+        if ((st = cu(cudaStreamSynchronize(s), "sync"))) return bail(st);
+    }
 
     // host: bucket table (R2, R7) and warp-task decomposition
     std::vector<long long> row_off((size_t)P * lf::kMaxT, -1);

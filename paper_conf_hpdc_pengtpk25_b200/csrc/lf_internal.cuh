@@ -3,6 +3,7 @@
 #pragma once
 
 #include <cuda_runtime.h>
+#include <stddef.h>
 #include <stdint.h>
 
 #include <string>
@@ -37,13 +38,14 @@ struct BucketDev {
 };
 
 // Stats the configure kernels accumulate (device, zero-initialised).
+struct StatsPart {
+    unsigned long long H[kMaxT], F[kMaxT], Unat[kMaxT], Utop[kMaxT];
+};
 struct StatsDev {
     unsigned long long len_min, len_max, len_sum, len_sumsq;  // row lengths
-    unsigned long long H[LF_MAX_PARTS][kMaxT];
-    unsigned long long F[LF_MAX_PARTS][kMaxT];
-    unsigned long long Unat[LF_MAX_PARTS][kMaxT];
-    unsigned long long Utop[LF_MAX_PARTS][kMaxT];
+    StatsPart part[LF_MAX_PARTS];  // only the first P are cleared / copied back
 };
+inline size_t stats_bytes(int P) { return offsetof(StatsDev, part) + (size_t)P * sizeof(StatsPart); }
 
 // ---- launchers (kernels in csrc/kernels/*.cu) ----
 uint32_t mask_slots(int64_t n_cols);  // words of the column-mask array (power of two >= K)

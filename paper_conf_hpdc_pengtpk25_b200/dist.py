@@ -78,8 +78,8 @@ def spmm_rowsharded(A_full, B: torch.Tensor, J: int, group=None, mode: str = "nn
     lo, hi = int(bounds[rank]), int(bounds[rank + 1])
     shard = Csr(A_full.row_ptr[lo:hi + 1], A_full.col_ind, A_full.val, A_full.n_cols,
                 int(rp_host[hi] - rp_host[lo]))
-    params, _ = configure(shard, J, **configure_kw)
-    M = CellMatrix.build(shard, params)
+    params, stats = configure(shard, J, **configure_kw)
+    M = CellMatrix.build(shard, params, stats)
     C_local = M.spmm(B)
     if not gather:
         return C_local, bounds

@@ -20,8 +20,8 @@ A = lf.Csr.from_host(A_h)
 B = torch.from_numpy(gen.dense(A_h.n_cols, J, 0)).cuda()
 C = torch.empty((A_h.n_rows, J), device="cuda")
 for _ in range(iters):
-    params, _ = lf.configure(A, J, **kw)
-    M = lf.CellMatrix.build(A, params)
+    params, stats = lf.configure(A, J, **kw)
+    M = lf.CellMatrix.build(A, params, stats)
     M.spmm(B, out=C)
     M.close()
 torch.cuda.synchronize()

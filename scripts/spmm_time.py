@@ -35,9 +35,9 @@ t = {"configure": [], "build": [], "spmm": []}
 for it in range(iters + 3):
     e0, e1, e2, e3 = ev(), ev(), ev(), ev()
     e0.record()
-    params, _ = lf.configure(A, J, **kw)
+    params, stats = lf.configure(A, J, **kw)
     e1.record()
-    M = lf.CellMatrix.build(A, params)
+    M = lf.CellMatrix.build(A, params, stats)
     e2.record()
     M.spmm(B, out=C)
     e3.record()

@@ -47,19 +47,19 @@ def test_null_arguments_rejected_on_host():
     """Host-side argument checks run before any CUDA call (works without a GPU)."""
     from paper_conf_hpdc_pengtpk25_b200 import _abi
     L = _abi.lib
-    assert L.lf_cell_build(None, None, None, None, None) == 1
+    assert L.lf_cell_build(None, None, None, None, None, None) == 1
     p = _abi.LfCellParams()
     p.n_parts = 0
     A = _abi.LfCsr(4, 4, 0, 8, 0, 0)
     h = ctypes.c_void_p()
-    assert L.lf_cell_build(ctypes.byref(A), ctypes.byref(p), None, None, ctypes.byref(h)) == 1
+    assert L.lf_cell_build(ctypes.byref(A), ctypes.byref(p), None, None, None, ctypes.byref(h)) == 1
     assert b"n_parts" in L.lf_last_error_detail()
     p.n_parts, p.use_cell = 1, 1
     p.max_width_log2[0], p.block_nnz_log2[0] = 3, 2
-    assert L.lf_cell_build(ctypes.byref(A), ctypes.byref(p), None, None, ctypes.byref(h)) == 1
+    assert L.lf_cell_build(ctypes.byref(A), ctypes.byref(p), None, None, None, ctypes.byref(h)) == 1
     A2 = _abi.LfCsr(1 << 28, 4, 0, 8, 0, 0)
     p.block_nnz_log2[0] = 3
-    assert L.lf_cell_build(ctypes.byref(A2), ctypes.byref(p), None, None, ctypes.byref(h)) == 3
+    assert L.lf_cell_build(ctypes.byref(A2), ctypes.byref(p), None, None, None, ctypes.byref(h)) == 3
     assert L.lf_spmm(None, None, 0, 4, None, 4, None) == 1
     assert L.lf_cell_configure(ctypes.byref(A), 0, None, ctypes.byref(p), None, None) == 1
 

@@ -112,6 +112,24 @@ def test_spmm_tolerance_float(lf, P, J):
     spmm_check(M, A_h, B_h)
 
 
+@pytest.mark.parametrize("P", [1, 3])
+def test_build_with_stats_equals_counted(lf, P):
+    """lf_cell_build with the configure statistics (no host sync) produces the
+    same arrays as the GPU-counted path, and both equal the oracle."""
+    A_h = gen.rmat(12, 16, seed=11)
+    A = lf.Csr.from_host(A_h)
+    params, stats = lf.configure(A, 64, force_parts=P)
+    M1 = lf.CellMatrix.build(A, params, stats)
+    M2 = lf.CellMatrix.build(A, params)
+    P_ = params.n_parts
+    cell = oracle.csr_to_cell(A_h, P_, list(params.max_width_log2[:P_]), list(params.block_nnz_log2[:P_]))
+    assert_cell_equal(M1, cell)
+    assert_cell_equal(M2, cell)
+    with pytest.raises(lf.LfError):
+        _, st1 = lf.configure(A, 64, force_parts=P + 1)
+        lf.CellMatrix.build(A, params, st1)
+
+
 def test_spmm_positive_gnn_style(lf):
     """All-positive values (val = 1, B in [0,1)): the adversarial case for the
     relative tolerance; long rows fold."""
@@ -219,8 +237,8 @@ FULL = ["c1_uniform1024", "c2_rmat20", "c3_stencil126"]
 def test_full_config_parity(lf, name):
     A_h, J = gen.config(name)
     A = lf.Csr.from_host(A_h)
-    params, _ = lf.configure(A, J)
-    M = lf.CellMatrix.build(A, params)
+    params, stats = lf.configure(A, J)
+    M = lf.CellMatrix.build(A, params, stats)  # the bench's path: sizes from the stats, no sync
     P = params.n_parts
     cell = oracle.csr_to_cell(A_h, P, list(params.max_width_log2[:P]), list(params.block_nnz_log2[:P]))
     assert_cell_equal(M, cell)
