@@ -62,6 +62,8 @@ def _L():
         _lib.lfgen_banded.argtypes = [ctypes.c_int64, ctypes.c_int64, ctypes.c_int64, ctypes.POINTER(_Csr)]
         _lib.lfgen_powerlaw.argtypes = [ctypes.c_int64, ctypes.c_int64, ctypes.c_double, ctypes.c_uint64,
                                         ctypes.POINTER(_Csr)]
+        _lib.lfgen_blockdiag.argtypes = [ctypes.c_int64, ctypes.c_int64, ctypes.POINTER(_Csr)]
+        _lib.lfgen_arrowhead.argtypes = [ctypes.c_int64, ctypes.c_int64, ctypes.POINTER(_Csr)]
         _lib.lfgen_fill_values.argtypes = [ctypes.c_void_p, ctypes.c_int64, ctypes.c_uint64, ctypes.c_uint64,
                                            ctypes.c_int32, ctypes.c_int32, ctypes.c_int32]
     return _lib
@@ -155,6 +157,41 @@ def powerlaw(n: int, total_nnz: int, sigma: float = 1.2, seed: int = 0, kind: in
     m = _Csr()
     rc = _L().lfgen_powerlaw(n, total_nnz, sigma, seed, ctypes.byref(m))
     return _take(m, rc, seed, kind, lo, hi, f"powerlaw{n}")
+
+
+def blockdiag(n: int, b: int, seed: int = 0, kind: int = GRID, lo: int = -3, hi: int = 3) -> CSR:
+    """Dense b x b diagonal blocks."""
+    m = _Csr()
+    rc = _L().lfgen_blockdiag(n, b, ctypes.byref(m))
+    return _take(m, rc, seed, kind, lo, hi, f"blockdiag{n}_{b}")
+
+
+def arrowhead(n: int, w: int, seed: int = 0, kind: int = GRID, lo: int = -3, hi: int = 3) -> CSR:
+    """w dense rows + w dense columns + the diagonal."""
+    m = _Csr()
+    rc = _L().lfgen_arrowhead(n, w, ctypes.byref(m))
+    return _take(m, rc, seed, kind, lo, hi, f"arrowhead{n}_{w}")
+
+
+def mixed_suite(sizes=(1 << 16, 1 << 18, 1 << 20), seeds=(0,)):
+    """BASELINE.json configs[4]: the mixed-skew suite --
+    yields (name, thunk) so callers generate one matrix at a time."""
+    for n in sizes:
+        sc = n.bit_length() - 1
+        for sd in seeds:
+            yield f"er_{n}_{sd}", (lambda n=n, sd=sd: uniform(n, n, 16.0 / n, sd))
+            for a in (0.45, 0.57, 0.70):
+                b = (1.0 - a) / 3.0 if a != 0.57 else 0.19
+                yield f"rmat{a}_{n}_{sd}", (lambda sc=sc, a=a, b=b, sd=sd: rmat(sc, 16, a, b, b, seed=sd))
+            for sg in (0.5, 1.0, 1.5, 2.0):
+                yield f"lognormal{sg}_{n}_{sd}", (lambda n=n, sg=sg, sd=sd: powerlaw(n, 16 * n, sg, sd))
+            for hw in (4, 16, 64):
+                yield f"band{hw}_{n}_{sd}", (lambda n=n, hw=hw, sd=sd: banded(n, hw, seed=sd))
+            g = round(n ** (1.0 / 3.0))
+            yield f"stencil27_{g}", (lambda g=g: stencil27(g))
+            for bb in (8, 32):
+                yield f"blockdiag{bb}_{n}", (lambda n=n, bb=bb: blockdiag(n, bb))
+            yield f"arrowhead_{n}", (lambda n=n: arrowhead(n, 4))
 
 
 def random_small(n_rows: int, n_cols: int, max_len: int, seed: int, dup: bool = True,

@@ -422,6 +422,57 @@ int lfgen_powerlaw(int64_t n, int64_t total_nnz, double sigma, uint64_t seed, lf
     return fail ? -1 : 0;
 }
 
+/* Block-diagonal: dense b x b blocks on the diagonal (n_rows = n_cols = n). */
+int lfgen_blockdiag(int64_t n, int64_t b, lfgen_csr *out) {
+    memset(out, 0, sizeof(*out));
+    if (n < 0 || b < 1) return -2;
+    out->n_rows = n;
+    out->n_cols = n;
+    out->row_ptr = (int64_t *)malloc((size_t)(n + 1) * sizeof(int64_t));
+    if (!out->row_ptr) return -1;
+    out->row_ptr[0] = 0;
+    for (int64_t i = 0; i < n; i++) {
+        int64_t lo = i / b * b, hi = lo + b < n ? lo + b : n;
+        out->row_ptr[i + 1] = out->row_ptr[i] + (hi - lo);
+    }
+    out->nnz = out->row_ptr[n];
+    out->col_ind = (int32_t *)malloc((size_t)(out->nnz > 0 ? out->nnz : 1) * sizeof(int32_t));
+    if (!out->col_ind) return -1;
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < n; i++) {
+        int64_t lo = i / b * b;
+        for (int64_t q = out->row_ptr[i]; q < out->row_ptr[i + 1]; q++) out->col_ind[q] = (int32_t)(lo + q - out->row_ptr[i]);
+    }
+    return 0;
+}
+
+/* Arrowhead: the first w rows and the first w columns are dense, plus the
+ * diagonal (n_rows = n_cols = n). */
+int lfgen_arrowhead(int64_t n, int64_t w, lfgen_csr *out) {
+    memset(out, 0, sizeof(*out));
+    if (n < 0 || w < 0 || w > n) return -2;
+    out->n_rows = n;
+    out->n_cols = n;
+    out->row_ptr = (int64_t *)malloc((size_t)(n + 1) * sizeof(int64_t));
+    if (!out->row_ptr) return -1;
+    out->row_ptr[0] = 0;
+    for (int64_t i = 0; i < n; i++) out->row_ptr[i + 1] = out->row_ptr[i] + (i < w ? n : w + (i >= w ? 1 : 0));
+    out->nnz = out->row_ptr[n];
+    out->col_ind = (int32_t *)malloc((size_t)(out->nnz > 0 ? out->nnz : 1) * sizeof(int32_t));
+    if (!out->col_ind) return -1;
+#pragma omp parallel for schedule(static)
+    for (int64_t i = 0; i < n; i++) {
+        int64_t q = out->row_ptr[i];
+        if (i < w) {
+            for (int64_t c = 0; c < n; c++) out->col_ind[q++] = (int32_t)c;
+        } else {
+            for (int64_t c = 0; c < w; c++) out->col_ind[q++] = (int32_t)c;
+            out->col_ind[q++] = (int32_t)i;
+        }
+    }
+    return 0;
+}
+
 /* Value fills.  kind:
  *   0: on the 2^-23 grid in [-1,1):   (u24 * 2^-23) - 1     (no denormals)
  *   1: integer in [lo,hi]                                   (exact-sum tests)
