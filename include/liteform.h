@@ -184,16 +184,32 @@ typedef struct lf_cell_arrays {
 typedef struct lf_cell lf_cell; /* opaque handle */
 
 /* Automatic composition (section 5, Fig. 2): computes the
- * statistics above on the GPU, decides use_cell and P (predictor slot,
- * sections 5.1-5.2; this build's rule is DESIGN.md "Predictor"), and for
- * each partition runs Algorithm 3 over eq. 7 (section 5.3) to pick e_p;
- * k_p = e_p + block_mult_log2.
+ * Table 2 features on the GPU, decides use_cell and P with lf_predict
+ * (sections 5.1-5.2) unless both are forced, then computes the per-partition
+ * statistics above and for each partition runs Algorithm 3 over eq. 7
+ * (section 5.3) to pick e_p; k_p = e_p + block_mult_log2.
  *   A      (host struct of device pointers)   J >= 1   opts may be NULL
  *   out    (host) receives the parameters     stats (host) may be NULL
- * Synchronises stream s once (one device-to-host copy of the statistics).
+ * Synchronises stream s twice when the predictor runs (features, then
+ * statistics: two small device-to-host copies), once otherwise.
  * Errors: LF_ERR_INVALID_ARG for bad sizes / pointers / options. */
 LF_API lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts *opts, lf_cell_params *out,
                             lf_configure_stats *stats, lf_stream_t s);
+
+/* LiteForm's predictors (sections 5.1-5.2), host only: from the
+ * Table 2/3 features -- features[8] = n_rows, n_cols,
+ * nnz, mean, min, max and population std of the row lengths, J, exactly as
+ * lf_configure_stats.features -- decide
+ *   *use_cell  1: CELL (Random Forest "CELL >= 1.1x faster than CSR",
+ *              P:L676-678); 0: the fixed-format CSR kernel (lf_csr_spmm)
+ *   *n_parts   column partitions P in {1, 2, 4, 8}, halved
+ *              until <= max_parts (0 = LF_MAX_PARTS).
+ * The forests were trained on B200 timings (scripts/train_predictor.py,
+ * profiles/r1_predictor.md); the paper ships no weights.
+ * Deterministic, no allocation, thread-safe.
+ * Errors: LF_ERR_INVALID_ARG (NULL pointer, negative / non-finite feature,
+ *         max_parts outside [0, LF_MAX_PARTS]). */
+LF_API lf_status lf_predict(const double features[8], int32_t max_parts, int32_t *use_cell, int32_t *n_parts);
 
 /* CSR -> CELL conversion on the GPU (section 4; canonical layout R1-R7; the
  * output is bit-identical to the oracle's).  Allocates the handle's arrays

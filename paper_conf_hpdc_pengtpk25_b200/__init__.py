@@ -24,7 +24,7 @@ from . import _abi
 from ._abi import (LF_MAX_PARTS, LfCsr, LfCellParams, LfConfigureOpts, LfConfigureStats, LfCellArrays,
                    LfError, lib)
 
-__all__ = ["Csr", "CellMatrix", "configure", "csr_spmm", "library_path", "LfError", "LF_MAX_PARTS"]
+__all__ = ["Csr", "CellMatrix", "configure", "predict", "csr_spmm", "library_path", "LfError", "LF_MAX_PARTS"]
 
 
 def library_path() -> str:
@@ -76,7 +76,8 @@ class Csr:
 def configure(A: Csr, J: int, *, max_parts: int = 0, block_mult_log2: int = 0, force_parts: int = 0,
               force_width_log2: int = -1, force_format: int = 0, stream=None):
     """Automatic CELL composition (section 5): returns
-    (LfCellParams, LfConfigureStats).  Synchronises the stream once."""
+    (LfCellParams, LfConfigureStats).  force_parts / force_format = 0 leave
+    P / the format to the predictor (lf_predict)."""
     opts = LfConfigureOpts(max_parts, block_mult_log2, force_parts, force_width_log2, force_format)
     params = LfCellParams()
     stats = LfConfigureStats()
@@ -84,6 +85,16 @@ def configure(A: Csr, J: int, *, max_parts: int = 0, block_mult_log2: int = 0, f
     _abi.check(lib.lf_cell_configure(ctypes.byref(csr), int(J), ctypes.byref(opts), ctypes.byref(params),
                                      ctypes.byref(stats), _stream(stream)))
     return params, stats
+
+
+def predict(features, max_parts: int = 0) -> tuple[int, int]:
+    """lf_predict (sections 5.1-5.2): (use_cell, P) from the 8 Table 2/3
+    features (n_rows, n_cols, nnz, mean, min, max, std of row lengths, J).
+    Host only; no GPU needed."""
+    f = (ctypes.c_double * 8)(*[float(x) for x in features])
+    u, p = ctypes.c_int32(), ctypes.c_int32()
+    _abi.check(lib.lf_predict(f, int(max_parts), ctypes.byref(u), ctypes.byref(p)))
+    return int(u.value), int(p.value)
 
 
 def make_params(n_parts: int, e, k=None, use_cell: int = 1) -> LfCellParams:

@@ -120,7 +120,7 @@ __global__ void __launch_bounds__(kThreads)
             // this segment holds all of row i's CELL rows and one warp sums them
             // (single CELL row, or a run of <= kMaxRun rows in a wide bucket);
             // F / L mark the first / last sub-row and are added below
-            const bool whole = row_cnt[i] == n_sub && (n_sub == 1 || (key >= 5 && n_sub <= kMaxRun));
+            const bool whole = row_cnt[i] == n_sub && key <= kPieceLog2 && (n_sub == 1 || (key >= 5 && n_sub <= kMaxRun));
             tag = (int32_t)((i << 3) | (whole ? 4 : 0));
             row_mode[i] = whole ? (n_sub == 1 ? kRowPlain : kRowRun) : kRowRed;
         }
@@ -272,7 +272,7 @@ __device__ __forceinline__ bool is_bound(const BucketDev *__restrict__ bk, int n
         if (bk[mid].task_off <= p) lo = mid;
         else hi = mid - 1;
     }
-    const int32_t tg = tag[bk[lo].row_off + (p - bk[lo].task_off)];
+    const int32_t tg = tag[bk[lo].row_off + ((p - bk[lo].task_off) >> bk[lo].piece_log2)];
     return tg < 0 || (tg & 2) || !(tg & 4);
 }
 

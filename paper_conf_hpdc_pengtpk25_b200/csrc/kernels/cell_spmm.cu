@@ -64,6 +64,11 @@ __device__ __forceinline__ float ld_stream(const float *p, uint64_t pol) {
     return v;
 }
 
+// Programmatic dependent launch: the SpMM kernel may start while
+// zero_rows_kernel (launched just before it, writing only the rows that later
+// receive red.add) is still running; a red waits for that grid first.
+__device__ __forceinline__ void grid_dep_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
 template <int VEC> struct Vec;
 template <> struct Vec<4> {
     using T = float4;
@@ -87,6 +92,7 @@ template <> struct Vec<4> {
                      : "memory");
     }
     static __device__ __forceinline__ void red(float *p, const T &v) {
+        grid_dep_wait();
         asm volatile("red.global.add.v4.f32 [%0], {%1, %2, %3, %4};" ::"l"(p), "f"(v.x), "f"(v.y), "f"(v.z),
                      "f"(v.w)
                      : "memory");
@@ -99,7 +105,10 @@ template <> struct Vec<1> {
     static __device__ __forceinline__ void fma(T &acc, float a, const T &b) { acc = fmaf(a, b, acc); }
     static __device__ __forceinline__ void add_xor(T &acc, int o) { acc += __shfl_xor_sync(kFull, acc, o); }
     static __device__ __forceinline__ void store(float *p, const T &v, uint64_t) { *p = v; }
-    static __device__ __forceinline__ void red(float *p, const T &v) { atomicAdd(p, v); }
+    static __device__ __forceinline__ void red(float *p, const T &v) {
+        grid_dep_wait();
+        atomicAdd(p, v);
+    }
 };
 
 // tag helpers
@@ -180,6 +189,9 @@ struct Ctx {
 // slot's B-row address (zero row for padding) and value, ordered so that lane
 // group g finds its steps k, k+1 (slots k*G+g, (k+1)*G+g) adjacent -- one
 // broadcast LDS.128 + one LDS.64 feed two gathers.
+#ifndef LF_RAWFETCH
+#define LF_RAWFETCH 1
+#endif
 struct Resolved {
     const float *addr[32];
     float val[32];
@@ -222,11 +234,28 @@ __device__ __forceinline__ void fetch(const Cx &cx, const Resolved &r, int kb, t
     }
 }
 
+// Same, straight from the cp.async-staged raw (col, val bits) pairs: one
+// broadcast LDS.128 feeds two gathers and the B-row address is formed in
+// registers (no resolve pass through shared memory).
+template <class Cx, int U>
+__device__ __forceinline__ void fetch(const Cx &cx, const int2 *raw, int kb, typename Cx::VT (&b)[U][Cx::NVv],
+                                      float (&a)[U]) {
+#pragma unroll
+    for (int u = 0; u < U; u += 2) {
+        const int p = cx.g * (32 / Cx::Gv) + kb + u;
+        const int4 e = *reinterpret_cast<const int4 *>(&raw[p]);
+        a[u] = __int_as_float(e.y);
+        cx.gather(cx.rowaddr(e.x), b[u]);
+        a[u + 1] = __int_as_float(e.w);
+        cx.gather(cx.rowaddr(e.z), b[u + 1]);
+    }
+}
+
 // the staged 32 slots accumulated into acc, no row boundary; slots at and
 // beyond n_real (a warp-uniform count: padding is a suffix of a CELL row)
 // are skipped a batch at a time
-template <class Cx>
-__device__ __forceinline__ void accum32(const Cx &cx, const Resolved &sw, typename Cx::VT (&acc)[Cx::NVv],
+template <class Cx, class Src>
+__device__ __forceinline__ void accum32(const Cx &cx, const Src &sw, typename Cx::VT (&acc)[Cx::NVv],
                                         int n_real = 32) {
     using V = typename Cx::V;
     using VT = typename Cx::VT;
@@ -247,8 +276,8 @@ __device__ __forceinline__ void accum32(const Cx &cx, const Resolved &sw, typena
 }
 
 // 32-slot task of a bucket with W = 2^T < 32: 32/W CELL rows, each written.
-template <class Cx, int T>
-__device__ __forceinline__ void narrow_task(const Cx &cx, const Resolved &sw, int32_t tag_l) {
+template <class Cx, int T, class Src>
+__device__ __forceinline__ void narrow_task(const Cx &cx, const Src &sw, int32_t tag_l) {
     using V = typename Cx::V;
     using VT = typename Cx::VT;
     constexpr int NV = Cx::NVv, G = Cx::Gv;
@@ -399,10 +428,16 @@ __device__ __forceinline__ void narrow_loop(const SpmmArgs &a, const Cx &cx0, Wa
         __syncwarp();
         const int32_t tag_l = st.tag[buf][lane];
         if (__ballot_sync(kFull, tag_l >= 0)) {
+#if LF_RAWFETCH
+            const int2 *sw = st.slot[buf];
+#else
             const Resolved &sw = st.res;
+#endif
             for (int j0 = 0; j0 < a.J; j0 += JT) {
                 cx.j0 = j0;
+#if !LF_RAWFETCH
                 resolve(cx, st.slot[buf], st.res, lane);
+#endif
                 switch (t) {
                 case 0: narrow_task<Cx, 0>(cx, sw, tag_l); break;
                 case 1: narrow_task<Cx, 1>(cx, sw, tag_l); break;
@@ -431,17 +466,19 @@ __device__ __forceinline__ void issue_wide(const SpmmArgs &a, const WideCursor &
                                            uint64_t pol, WarpStage &st, int buf) {
     const BucketDev *bk = a.bk_w + bcur;
     const int64_t tin = c.task - __ldg(&bk->task_off);
-    const int64_t s = __ldg(&bk->slot_off) + (tin << __ldg(&bk->t)) + 32 * c.k + lane;
+    const int pl = __ldg(&bk->piece_log2);  // task = piece (tin & (2^pl - 1)) of CELL row tin >> pl
+    const int64_t s = __ldg(&bk->slot_off) + ((tin >> pl) << __ldg(&bk->t)) + ((tin & ((1 << pl) - 1)) << kPieceLog2) +
+                      32 * c.k + lane;
     int2 *dst = &st.slot[buf][stage_pos<G>(lane)];
     cp_async4(&dst->x, a.col + s, pol);
     cp_async4(&dst->y, a.val + s, pol);
-    if (c.k == 0 && lane == 0) cp_async4(&st.tag[buf][0], a.row_tag + __ldg(&bk->row_off) + tin, pol);
+    if (c.k == 0 && lane == 0) cp_async4(&st.tag[buf][0], a.row_tag + __ldg(&bk->row_off) + (tin >> pl), pol);
     cp_commit();
 }
 
 __device__ __forceinline__ int wide_nch(const SpmmArgs &a, int64_t task, int &bcur) {
     while (bcur + 1 < a.nb_w && __ldg(&a.bk_w[bcur + 1].task_off) <= task) bcur++;
-    return 1 << (__ldg(&a.bk_w[bcur].t) - 5);
+    return 1 << (min(__ldg(&a.bk_w[bcur].t), kPieceLog2) - 5);
 }
 
 // Run-aligned claims: a claimed range [x, x + size) of the wide class really
@@ -542,8 +579,12 @@ __device__ __forceinline__ void wide_loop(const SpmmArgs &a, const Cx &cx, WarpS
         }
         const int n_real = row_tag >= 0 ? __popc(__ballot_sync(kFull, st.slot[buf][stage_pos<G>(lane)].x >= 0)) : 0;
         if (n_real > 0) {
+#if LF_RAWFETCH
+            accum32(cx, (const int2 *)st.slot[buf], acc, n_real);
+#else
             resolve(cx, st.slot[buf], st.res, lane);
             accum32(cx, st.res, acc, n_real);
+#endif
         }
         if (cur.k == cur.nch - 1) {
 #ifdef LF_TRACE
@@ -587,9 +628,11 @@ __device__ __forceinline__ void wide_loop_tiled(const SpmmArgs &a, const Cx &cx0
             const int nch = wide_nch(a, task, bcur);
             const BucketDev *bk = a.bk_w + bcur;
             const int64_t tin = task - __ldg(&bk->task_off);
-            const int32_t tag = __ldg(a.row_tag + __ldg(&bk->row_off) + tin);
+            const int pl = __ldg(&bk->piece_log2);
+            const int32_t tag = __ldg(a.row_tag + __ldg(&bk->row_off) + (tin >> pl));
             if (tag < 0) continue;
-            const int64_t s0 = __ldg(&bk->slot_off) + (tin << __ldg(&bk->t));
+            const int64_t s0 = __ldg(&bk->slot_off) + ((tin >> pl) << __ldg(&bk->t)) +
+                               ((tin & ((1 << pl) - 1)) << kPieceLog2);
             for (int j0 = 0; j0 < a.J; j0 += JT) {
                 cx.j0 = j0;
                 VT acc[NV];
@@ -612,8 +655,12 @@ __device__ __forceinline__ void wide_loop_tiled(const SpmmArgs &a, const Cx &cx0
 // W >= 32 queue; a warp whose queue is drained helps with the other one.
 // The two loops run one after the other (no live state in common), so each
 // is register-allocated alone.  Epilogue: empty C rows are zeroed.
+// resident blocks per SM: wider J slices per lane (NV float4) need more
+// registers for the accumulators and the gathers in flight (no spills)
+constexpr int min_blocks(int NV) { return NV >= 4 ? 2 : NV == 2 ? 3 : kMinBlocks; }
+
 template <int VEC, int G, int NV, bool FULL>
-__global__ void __launch_bounds__(kWarpsPerBlock * 32, kMinBlocks) cell_spmm_kernel(const SpmmArgs a) {
+__global__ void __launch_bounds__(kWarpsPerBlock * 32, min_blocks(NV)) cell_spmm_kernel(const SpmmArgs a) {
     using Cx = Ctx<VEC, G, NV, FULL>;
     using L = Layout<VEC, G, NV>;
     __shared__ __align__(16) WarpStage stage_buf[kWarpsPerBlock];
@@ -647,6 +694,17 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, kMinBlocks) cell_spmm_ker
     if (LF_EPI_ZERO)
         zero_rows_warp(a.row_mode, a.n_rows, a.C, a.ldc, a.J, VEC == 4, 1u << kRowEmpty,
                        (int64_t)blockIdx.x * kWarpsPerBlock + w, (int64_t)gridDim.x * kWarpsPerBlock, lane, pol);
+    // the last warp out resets the queue counters for the next launch that
+    // uses this slot (every claim of every warp is ordered before its fence)
+    if (lane == 0) {
+        __threadfence();
+        if (atomicAdd(a.ctr + 2, 1ull) == (unsigned long long)gridDim.x * kWarpsPerBlock - 1) {
+            __threadfence();
+            a.ctr[0] = 0;
+            a.ctr[1] = 0;
+            a.ctr[2] = 0;
+        }
+    }
 #ifdef LF_TRACE
     if (lane == 0) lf_trace_buf[(blockIdx.x * kWarpsPerBlock + w) * 2] = t_work;
     unsigned long long t_end;
@@ -691,6 +749,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32)
 
 __global__ void zero_rows_kernel(const uint8_t *__restrict__ row_mode, int64_t n_rows, float *__restrict__ C,
                                  int64_t ldc, int J, int vec4, unsigned mode_mask) {
+    asm volatile("griddepcontrol.launch_dependents;");
     const int lane = threadIdx.x & 31;
     const int64_t gwarp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
@@ -727,15 +786,19 @@ cudaError_t run_cell(const SpmmArgs &a0, cudaStream_t s) {
     const int64_t want_z = std::min<int64_t>(cap, (a.n_rows + 32 * kWarpsPerBlock - 1) / (32 * kWarpsPerBlock));
     const int grid = (int)std::max<int64_t>(bn + bw, want_z);
     if (grid == 0) return cudaSuccess;
-    // per-launch queue counters (stream-ordered), so concurrent calls on one
-    // handle stay independent
-    unsigned long long *ctr = nullptr;
-    cudaError_t e = cudaMallocAsync(&ctr, 2 * sizeof(unsigned long long), s);
+    // a.ctr: the handle's counter slot for this launch (zero; reset by the
+    // kernel's last warp)
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)grid);
+    cfg.blockDim = dim3(kWarpsPerBlock * 32);
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;  // overlap zero_rows_kernel
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, fn, a);
     if (e != cudaSuccess) return e;
-    if ((e = cudaMemsetAsync(ctr, 0, 2 * sizeof(unsigned long long), s)) != cudaSuccess) return e;
-    a.ctr = ctr;
-    fn<<<grid, kWarpsPerBlock * 32, 0, s>>>(a);
-    if ((e = cudaGetLastError()) != cudaSuccess) return e;
 #ifdef LF_TRACE
     {
         static std::vector<unsigned long long> h(2 * 148 * 64);
@@ -769,7 +832,7 @@ cudaError_t run_cell(const SpmmArgs &a0, cudaStream_t s) {
                 nw, a.blocks_n, wk[0], wk[nw / 10], wk[nw / 2], wk[nw * 9 / 10], wk[nw - 1], en[nw / 2], en[nw - 1]);
     }
 #endif
-    return cudaFreeAsync(ctr, s);
+    return cudaSuccess;
 }
 
 template <int VEC, int G, int NV>

@@ -102,13 +102,19 @@ lf_status maybe_validate(const lf_csr *A, cudaStream_t s) {
     return LF_OK;
 }
 
-// Predictor slot (sections 5.1-5.2).  No trained model exists
-// for this hardware (parity unpinned): the stand-in
-// chooses CELL and P = 1.
-int standin_parts(const lf_csr *A, int32_t J, int max_parts) {
-    (void)A;
-    (void)J;
-    return std::max(1, std::min(1, max_parts));
+// Table 2 + Table 3's J from the row-length sums
+void table2_features(const lf_csr &A, int32_t J, const lf::StatsDev &st, double f[8]) {
+    const double I = (double)A.n_rows;
+    const double mean = A.n_rows ? (double)st.len_sum / I : 0.0;
+    const double var = A.n_rows ? (double)st.len_sumsq / I - mean * mean : 0.0;
+    f[0] = I;
+    f[1] = (double)A.n_cols;
+    f[2] = (double)st.len_sum;
+    f[3] = mean;
+    f[4] = A.n_rows ? (double)st.len_min : 0.0;
+    f[5] = (double)st.len_max;
+    f[6] = var > 0 ? std::sqrt(var) : 0.0;
+    f[7] = (double)J;
 }
 
 // Algorithm 3 in exponent space (reading R8) over eq. 7 costs.
@@ -161,7 +167,29 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
     if (lf_status st = maybe_validate(A, s)) return st;
 
     keep_default_pool();
-    const int P = o.force_parts ? o.force_parts : standin_parts(A, J, max_parts);
+    // pinned staging buffer (one per thread) so the copies back are plain DMAs
+    thread_local lf::StatsDev *h_st = nullptr;
+    if (!h_st) LF_CUDA(cudaMallocHost(&h_st, sizeof(lf::StatsDev)));
+    // predictor (sections 5.1-5.2): Table 2 features first, then format and P
+    int P = o.force_parts;
+    int use_cell = o.force_format == 2 ? 0 : 1;
+    if (o.force_parts == 0 || o.force_format == 0) {
+        lf::StatsDev *d_f = nullptr;
+        const size_t fb = lf::stats_bytes(0);
+        LF_CUDA(cudaMallocAsync(&d_f, fb, s));
+        LF_CUDA(cudaMemsetAsync(d_f, 0, fb, s));
+        LF_CUDA(cudaMemsetAsync(&d_f->len_min, 0xFF, sizeof(unsigned long long), s));
+        LF_CUDA(lf::launch_features(*A, d_f, s));
+        LF_CUDA(cudaMemcpyAsync(h_st, d_f, fb, cudaMemcpyDeviceToHost, s));
+        LF_CUDA(cudaFreeAsync(d_f, s));
+        LF_CUDA(cudaStreamSynchronize(s));
+        double f[8];
+        table2_features(*A, J, *h_st, f);
+        int32_t pu = 1, pp = 1;
+        if (lf_status st = lf_predict(f, max_parts, &pu, &pp)) return fail(st, "lf_predict");
+        if (o.force_format == 0) use_cell = pu;
+        if (o.force_parts == 0) P = pp;
+    }
     lf::StatsDev *d_st = nullptr;
     uint32_t *d_mask = nullptr;
     const size_t st_bytes = lf::stats_bytes(P);
@@ -176,9 +204,6 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
     uint8_t *d_t0 = nullptr;
     if (A->n_rows > 0) LF_CUDA(cudaMallocAsync(&d_t0, lf::stats_scratch_bytes(A->n_rows, A->nnz, P), s));
     LF_CUDA(lf::launch_stats(*A, P, d_st, d_mask, d_t0, s));
-    // pinned staging buffer (one per thread) so the copy back is a plain DMA
-    thread_local lf::StatsDev *h_st = nullptr;
-    if (!h_st) LF_CUDA(cudaMallocHost(&h_st, sizeof(lf::StatsDev)));
     LF_CUDA(cudaMemcpyAsync(h_st, d_st, st_bytes, cudaMemcpyDeviceToHost, s));
     LF_CUDA(cudaFreeAsync(d_st, s));
     if (d_mask) LF_CUDA(cudaFreeAsync(d_mask, s));
@@ -189,21 +214,11 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
     lf_configure_stats local;
     lf_configure_stats &cs = stats ? *stats : local;
     std::memset(&cs, 0, sizeof(cs));
-    const double I = (double)A->n_rows;
-    const double mean = A->n_rows ? (double)st.len_sum / I : 0.0;
-    double var = A->n_rows ? (double)st.len_sumsq / I - mean * mean : 0.0;
-    cs.features[0] = I;
-    cs.features[1] = (double)A->n_cols;
-    cs.features[2] = (double)st.len_sum;
-    cs.features[3] = mean;
-    cs.features[4] = A->n_rows ? (double)st.len_min : 0.0;
-    cs.features[5] = (double)st.len_max;
-    cs.features[6] = var > 0 ? std::sqrt(var) : 0.0;
-    cs.features[7] = (double)J;
+    table2_features(*A, J, st, cs.features);
     cs.n_parts = P;
 
     lf_cell_params prm{};
-    prm.use_cell = o.force_format == 2 ? 0 : 1;
+    prm.use_cell = use_cell;
     prm.n_parts = P;
     for (int p = 0; p < P; p++) {
         int top = -1;
@@ -349,7 +364,8 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
             d.row_off = R_tot;
             d.n_slots = pad * W;
             d.t = t;
-            d.task_slots = (int32_t)std::max<int64_t>(32, W);
+            d.piece_log2 = std::max(0, t - lf::kPieceLog2);
+            d.task_slots = (int32_t)std::max<int64_t>(32, W >> d.piece_log2);
             if (W < 32) {
                 d.task_off = h->n_tasks_n;
                 h->n_tasks_n += (pad * W + 31) / 32;
@@ -357,7 +373,7 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
                 bn.push_back(d);
             } else {
                 d.task_off = h->n_tasks_w;
-                h->n_tasks_w += pad;
+                h->n_tasks_w += pad << d.piece_log2;
                 h->slots_w += pad * W;
                 bw.push_back(d);
             }
@@ -382,8 +398,8 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
     auto up = [&](size_t b) { return (b + a256 - 1) / a256 * a256; };
     const size_t b_ri = up(R_tot * 4), b_rt = up(R_tot * 4), b_ci = up(S_tot * 4), b_va = up(S_tot * 4),
                  b_bk = up(h->h_buckets.size() * sizeof(lf::BucketDev)),
-                 b_rb = up((size_t)(h->n_tasks_w + 1));
-    h->pool_bytes = b_ri + b_rt + b_ci + b_va + b_bk + b_rb;
+                 b_rb = up((size_t)(h->n_tasks_w + 1)), b_ct = up(kCtrSlots * 4 * sizeof(unsigned long long));
+    h->pool_bytes = b_ri + b_rt + b_ci + b_va + b_bk + b_rb + b_ct;
     h->pool = mem.get(h->pool_bytes);
     if (h->pool_bytes && !h->pool) return bail(fail(LF_ERR_NO_MEMORY, "CELL arrays allocation failed"));
     char *q = static_cast<char *>(h->pool);
@@ -393,6 +409,8 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
     h->val = reinterpret_cast<float *>(q + b_ri + b_rt + b_ci);
     h->d_buckets = reinterpret_cast<lf::BucketDev *>(q + b_ri + b_rt + b_ci + b_va);
     h->run_bound = reinterpret_cast<uint8_t *>(q + b_ri + b_rt + b_ci + b_va + b_bk);
+    h->ctr_ring = reinterpret_cast<unsigned long long *>(q + b_ri + b_rt + b_ci + b_va + b_bk + b_rb);
+    if ((st = cu(cudaMemsetAsync(h->ctr_ring, 0, b_ct, s), "memset"))) return bail(st);
     bs.src_pos = sc.get<int64_t>((size_t)R_tot);
     bs.src_cnt = sc.get<int32_t>((size_t)R_tot);
     if (R_tot && (!bs.src_pos || !bs.src_cnt)) return bail(fail(LF_ERR_NO_MEMORY, "scratch allocation failed"));
@@ -439,7 +457,8 @@ lf_status lf_spmm(const lf_cell *h, const float *B, int64_t ldb, int32_t J, floa
     }
     const int nb = (int)h->buckets.size();
     lf::SpmmArgs a{h->d_buckets + nb, h->d_buckets + nb + h->nb_n, h->nb_n, h->nb_w, h->n_tasks_n, h->n_tasks_w,
-                   h->slots_n, h->slots_w, 0, h->row_mode, h->n_rows, h->run_bound, nullptr, h->col_ind, h->val,
+                   h->slots_n, h->slots_w, 0, h->row_mode, h->n_rows, h->run_bound,
+                   h->ctr_ring + 4 * (h->launch_seq.fetch_add(1, std::memory_order_relaxed) % kCtrSlots), h->col_ind, h->val,
                    h->row_tag,
                    B, ldb, C, ldc, J};
     LF_CUDA(lf::launch_cell_spmm(a, s));

@@ -7,6 +7,7 @@
 #include <stdint.h>
 
 #include <string>
+#include <atomic>
 #include <vector>
 
 #include "liteform.h"
@@ -34,7 +35,9 @@ struct BucketDev {
     int64_t n_slots;    // n_rows_pad * W
     int64_t task_off;   // first task index of this bucket
     int32_t t;          // log2 width
-    int32_t task_slots; // slots per task: 32 (W <= 32) or W (one row per task)
+    int32_t task_slots; // slots per task: 32 (W <= 32), W (W <= 2^kPieceLog2) or 2^kPieceLog2
+    int32_t piece_log2; // W >= 32: a CELL row is 2^piece_log2 tasks of <= 2^kPieceLog2 slots
+    int32_t pad_;
 };
 
 // Stats the configure kernels accumulate (device, zero-initialised).
@@ -50,6 +53,7 @@ inline size_t stats_bytes(int P) { return offsetof(StatsDev, part) + (size_t)P *
 // ---- launchers (kernels in csrc/kernels/*.cu) ----
 uint32_t mask_slots(int64_t n_cols);  // words of the column-mask array (power of two >= K)
 size_t stats_scratch_bytes(int64_t n_rows, int64_t nnz, int P);  // t0 per segment + tile -> row map
+cudaError_t launch_features(const lf_csr &A, StatsDev *d_stats, cudaStream_t s);  // len_* only
 cudaError_t launch_stats(const lf_csr &A, int P, StatsDev *d_stats, uint32_t *d_colmask, uint8_t *d_t0seg,
                          cudaStream_t s);
 
@@ -76,6 +80,14 @@ constexpr int kMaxRun = LF_MAX_RUN;
 #define LF_WIDE_CHUNK 8
 #endif
 constexpr int kWideChunk = LF_WIDE_CHUNK;
+// A CELL row wider than 2^kPieceLog2 slots (a large max width chosen by
+// Algorithm 3, e.g. the dense rows of an arrowhead matrix) is split into
+// pieces of 2^kPieceLog2 slots, separate wide tasks that red.add into the
+// pre-zeroed C row, so one long row never serialises on a single warp.
+#ifndef LF_PIECE_LOG2
+#define LF_PIECE_LOG2 10
+#endif
+constexpr int kPieceLog2 = LF_PIECE_LOG2;
 // row_mode[i]: how C row i is produced
 enum : uint8_t {
     kRowPlain = 0,  // one CELL row, plain store
@@ -107,7 +119,7 @@ struct SpmmArgs {
     const uint8_t *row_mode;
     int64_t n_rows;
     const uint8_t *run_bound;  // [n_tasks_w + 1]
-    unsigned long long *ctr;   // per-launch work-queue counters (set by the launcher)
+    unsigned long long *ctr;   // [4] the handle's counter slot for this launch: wide, narrow, warps done
     const int32_t *col;
     const float *val;
     const int32_t *row_tag;
@@ -124,6 +136,7 @@ cudaError_t launch_validate(const lf_csr &A, int *d_flag, cudaStream_t s);
 
 }  // namespace lf
 
+constexpr int kCtrSlots = 64;  // concurrent lf_spmm launches on one handle
 struct lf_cell {
     lf_cell_params params;
     int64_t n_rows = 0, n_cols = 0, nnz = 0;
@@ -137,6 +150,11 @@ struct lf_cell {
     uint8_t *row_mode = nullptr;  // [n_rows] kRow* (how each C row is produced)
     uint8_t *run_bound = nullptr; // [n_tasks_w + 1] (in the pool)
     lf::BucketDev *d_buckets = nullptr;  // [nb] all, then [nb_n] W < 32 class, then [nb_w] W >= 32 class
+    // work-queue counters, kCtrSlots slots of 4 (wide, narrow, warps done, -)
+    // in the pool: launch k uses slot k % kCtrSlots and its last warp resets
+    // it, so lf_spmm needs no allocation or memset per call
+    unsigned long long *ctr_ring = nullptr;
+    mutable std::atomic<uint32_t> launch_seq{0};
     std::vector<lf_bucket> buckets;
     std::vector<lf::BucketDev> h_buckets;
     // memory: one pool allocation holds every array above

@@ -238,6 +238,10 @@ def test_full_config_parity(lf, name):
     A_h, J = gen.config(name)
     A = lf.Csr.from_host(A_h)
     params, stats = lf.configure(A, J)
+    # the predictor's decision is the one lf_predict makes on the same features
+    assert (params.use_cell, params.n_parts) == lf.predict(list(stats.features))
+    if params.use_cell == 0:  # fixed CSR format chosen: check CELL at the predicted P too
+        params, stats = lf.configure(A, J, force_parts=params.n_parts, force_format=1)
     M = lf.CellMatrix.build(A, params, stats)  # the bench's path: sizes from the stats, no sync
     P = params.n_parts
     cell = oracle.csr_to_cell(A_h, P, list(params.max_width_log2[:P]), list(params.block_nnz_log2[:P]))
@@ -263,3 +267,46 @@ def test_full_reddit_parity(lf):
     # builder: the arrays of the 20 longest rows' buckets via the round-trip
     v = M.view()
     assert int(v["n_slots"]) >= A_h.nnz
+
+
+@pytest.mark.parametrize("width", [None, 12])
+def test_long_rows_split_into_pieces(lf, width):
+    """Rows wider than 2^kPieceLog2 = 1024 slots (the dense rows of an
+    arrowhead matrix, Algorithm 3 picks W = 2^14 here; or a forced 2^12 on
+    R-MAT) are processed as several wide tasks that red.add into the row:
+    the CELL arrays are unchanged and C stays within tolerance."""
+    if width is None:
+        A_h = gen.arrowhead(1 << 14, 4, seed=1)
+        kw = dict(force_parts=1, force_format=1)
+    else:
+        A_h = gen.rmat(14, 16, seed=4)
+        kw = dict(force_parts=1, force_format=1, force_width_log2=width)
+    A = lf.Csr.from_host(A_h)
+    for J in (64, 128, 512, 640):
+        params, stats = lf.configure(A, J, **kw)
+        assert params.max_width_log2[0] > 10
+        M = lf.CellMatrix.build(A, params, stats)
+        cell = oracle.csr_to_cell(A_h, 1, [params.max_width_log2[0]], [params.block_nnz_log2[0]])
+        assert_cell_equal(M, cell)
+        spmm_check(M, A_h, gen.dense(A_h.n_cols, J, 7))
+
+
+def test_repeated_launches_reuse_counter_slots(lf):
+    """More launches than the handle's counter ring (64 slots, each reset by
+    its kernel's last warp), on two streams: every result stays correct."""
+    A_h = gen.rmat(12, 16, seed=3, kind=gen.INT)
+    B_h = gen.dense(A_h.n_cols, 64, 3, gen.INT)
+    A = lf.Csr.from_host(A_h)
+    M = lf.CellMatrix.build(A, lf.make_params(1, 4))
+    B = torch.from_numpy(B_h).cuda()
+    ref = oracle.spmm_csr(A_h, B_h)[0]
+    s2 = torch.cuda.Stream()
+    torch.cuda.synchronize()
+    outs = []
+    for it in range(150):
+        st = s2 if it % 3 == 0 else torch.cuda.current_stream()
+        with torch.cuda.stream(st):
+            outs.append(M.spmm(B, stream=st))
+    torch.cuda.synchronize()
+    for C in outs[::7] + outs[-3:]:
+        assert np.array_equal(C.cpu().numpy().astype(np.float64), ref)
