@@ -187,6 +187,11 @@ def mixed_suite(sizes=(1 << 16, 1 << 18, 1 << 20), seeds=(0,)):
                 yield f"lognormal{sg}_{n}_{sd}", (lambda n=n, sg=sg, sd=sd: powerlaw(n, 16 * n, sg, sd))
             for hw in (4, 16, 64):
                 yield f"band{hw}_{n}_{sd}", (lambda n=n, hw=hw, sd=sd: banded(n, hw, seed=sd))
+            # GNN-degree lognormal graphs (Reddit-shaped, mean degree 128 / 512 over
+            # n/4 rows): the regime where B outgrows L2 and rows are long enough
+            # for column partitions (P > 1) to pay off
+            for deg in (128, 512):
+                yield f"gnn{deg}_{n}_{sd}", (lambda n=n, deg=deg, sd=sd: powerlaw(n // 4, deg * (n // 4), 1.2, sd))
             g = round(n ** (1.0 / 3.0))
             yield f"stencil27_{g}", (lambda g=g: stencil27(g))
             for bb in (8, 32):

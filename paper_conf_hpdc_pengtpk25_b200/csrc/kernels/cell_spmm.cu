@@ -189,9 +189,6 @@ struct Ctx {
 // slot's B-row address (zero row for padding) and value, ordered so that lane
 // group g finds its steps k, k+1 (slots k*G+g, (k+1)*G+g) adjacent -- one
 // broadcast LDS.128 + one LDS.64 feed two gathers.
-#ifndef LF_RAWFETCH
-#define LF_RAWFETCH 1
-#endif
 struct Resolved {
     const float *addr[32];
     float val[32];
@@ -234,28 +231,11 @@ __device__ __forceinline__ void fetch(const Cx &cx, const Resolved &r, int kb, t
     }
 }
 
-// Same, straight from the cp.async-staged raw (col, val bits) pairs: one
-// broadcast LDS.128 feeds two gathers and the B-row address is formed in
-// registers (no resolve pass through shared memory).
-template <class Cx, int U>
-__device__ __forceinline__ void fetch(const Cx &cx, const int2 *raw, int kb, typename Cx::VT (&b)[U][Cx::NVv],
-                                      float (&a)[U]) {
-#pragma unroll
-    for (int u = 0; u < U; u += 2) {
-        const int p = cx.g * (32 / Cx::Gv) + kb + u;
-        const int4 e = *reinterpret_cast<const int4 *>(&raw[p]);
-        a[u] = __int_as_float(e.y);
-        cx.gather(cx.rowaddr(e.x), b[u]);
-        a[u + 1] = __int_as_float(e.w);
-        cx.gather(cx.rowaddr(e.z), b[u + 1]);
-    }
-}
-
 // the staged 32 slots accumulated into acc, no row boundary; slots at and
 // beyond n_real (a warp-uniform count: padding is a suffix of a CELL row)
 // are skipped a batch at a time
-template <class Cx, class Src>
-__device__ __forceinline__ void accum32(const Cx &cx, const Src &sw, typename Cx::VT (&acc)[Cx::NVv],
+template <class Cx>
+__device__ __forceinline__ void accum32(const Cx &cx, const Resolved &sw, typename Cx::VT (&acc)[Cx::NVv],
                                         int n_real = 32) {
     using V = typename Cx::V;
     using VT = typename Cx::VT;
@@ -276,8 +256,8 @@ __device__ __forceinline__ void accum32(const Cx &cx, const Src &sw, typename Cx
 }
 
 // 32-slot task of a bucket with W = 2^T < 32: 32/W CELL rows, each written.
-template <class Cx, int T, class Src>
-__device__ __forceinline__ void narrow_task(const Cx &cx, const Src &sw, int32_t tag_l) {
+template <class Cx, int T>
+__device__ __forceinline__ void narrow_task(const Cx &cx, const Resolved &sw, int32_t tag_l) {
     using V = typename Cx::V;
     using VT = typename Cx::VT;
     constexpr int NV = Cx::NVv, G = Cx::Gv;
@@ -428,16 +408,10 @@ __device__ __forceinline__ void narrow_loop(const SpmmArgs &a, const Cx &cx0, Wa
         __syncwarp();
         const int32_t tag_l = st.tag[buf][lane];
         if (__ballot_sync(kFull, tag_l >= 0)) {
-#if LF_RAWFETCH
-            const int2 *sw = st.slot[buf];
-#else
             const Resolved &sw = st.res;
-#endif
             for (int j0 = 0; j0 < a.J; j0 += JT) {
                 cx.j0 = j0;
-#if !LF_RAWFETCH
                 resolve(cx, st.slot[buf], st.res, lane);
-#endif
                 switch (t) {
                 case 0: narrow_task<Cx, 0>(cx, sw, tag_l); break;
                 case 1: narrow_task<Cx, 1>(cx, sw, tag_l); break;
@@ -579,12 +553,8 @@ __device__ __forceinline__ void wide_loop(const SpmmArgs &a, const Cx &cx, WarpS
         }
         const int n_real = row_tag >= 0 ? __popc(__ballot_sync(kFull, st.slot[buf][stage_pos<G>(lane)].x >= 0)) : 0;
         if (n_real > 0) {
-#if LF_RAWFETCH
-            accum32(cx, (const int2 *)st.slot[buf], acc, n_real);
-#else
             resolve(cx, st.slot[buf], st.res, lane);
             accum32(cx, st.res, acc, n_real);
-#endif
         }
         if (cur.k == cur.nch - 1) {
 #ifdef LF_TRACE

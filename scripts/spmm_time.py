@@ -20,6 +20,8 @@ if "parts" in opt:
     kw["force_parts"] = int(opt["parts"])
 if "width" in opt:
     kw["force_width_log2"] = int(opt["width"])
+if "fmt" in opt:
+    kw["force_format"] = int(opt["fmt"])
 if "mult" in opt:
     kw["block_mult_log2"] = int(opt["mult"])
 A_h, J = gen.config(cfg)
