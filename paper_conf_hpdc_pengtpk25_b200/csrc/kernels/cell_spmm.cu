@@ -39,6 +39,12 @@ namespace {
 
 constexpr unsigned kFull = 0xffffffffu;
 constexpr int kWarpsPerBlock = 8;
+#ifndef LF_SKIP_PAD
+#define LF_SKIP_PAD 0  // measured: the per-slot predicate costs more than the skipped zero-row loads
+#endif
+#ifndef LF_ZERO_FIRST
+#define LF_ZERO_FIRST 1  // empty rows zeroed before the gathers (overlapped), not in a tail phase
+#endif
 #ifndef LF_EPI_ZERO
 #define LF_EPI_ZERO 1  // empty C rows zeroed in the SpMM kernel's epilogue
 #endif
@@ -159,8 +165,14 @@ struct Ctx {
         return c >= 0 ? B + (int64_t)c * ldb : reinterpret_cast<const float *>(g_zero_row) - j0;
     }
     __device__ __forceinline__ void gather(const float *r, VT (&b)[NV]) const {
+#if LF_SKIP_PAD
+        // a padding slot (zero-row address) issues no load at all
+        const bool real = r != reinterpret_cast<const float *>(g_zero_row) - j0;
+#else
+        const bool real = true;
+#endif
 #pragma unroll
-        for (int m = 0; m < NV; m++) b[m] = jok(m) ? V::load(r + jcol(m)) : V::zero();
+        for (int m = 0; m < NV; m++) b[m] = (jok(m) && real) ? V::load(r + jcol(m)) : V::zero();
     }
     // write one C row slice: plain store when this write is the row's only one
     __device__ __forceinline__ void write(int32_t row, bool plain, const VT (&acc)[NV]) const {
@@ -168,6 +180,9 @@ struct Ctx {
 #pragma unroll
         for (int m = 0; m < NV; m++) {
             if (!jok(m)) continue;
+#ifdef LF_DIAG_NOWRITE  // diagnostic builds only: drop the C traffic
+            if (reinterpret_cast<const float *>(&acc[m])[0] != 1234.5f) continue;
+#endif
             if (plain) V::store(p + jcol(m), acc[m], pol);
             else V::red(p + jcol(m), acc[m]);
         }
@@ -648,6 +663,17 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, min_blocks(NV)) cell_spmm
     }
 #endif
     const int64_t nw = (int64_t)gridDim.x * kWarpsPerBlock;
+#ifdef LF_DIAG_NOWRITE
+    constexpr bool kZero = false;
+#else
+    constexpr bool kZero = LF_EPI_ZERO;
+#endif
+    // rows of A with no CELL row are written +0.0 (R13) by every warp for its
+    // share of the rows; done first, the write traffic overlaps the gathers
+    // of the warps already streaming instead of forming a tail phase
+    if (kZero && LF_ZERO_FIRST)
+        zero_rows_warp(a.row_mode, a.n_rows, a.C, a.ldc, a.J, VEC == 4, 1u << kRowEmpty,
+                       (int64_t)blockIdx.x * kWarpsPerBlock + w, nw, lane, pol);
     if ((int)blockIdx.x < a.blocks_n) {
         narrow_loop(a, cx, st, lane, nw, pol);
         if (tiled) wide_loop_tiled(a, cx, st, lane, pol);
@@ -661,7 +687,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, min_blocks(NV)) cell_spmm
     unsigned long long t_work;
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_work));
 #endif
-    if (LF_EPI_ZERO)
+    if (kZero && !LF_ZERO_FIRST)
         zero_rows_warp(a.row_mode, a.n_rows, a.C, a.ldc, a.J, VEC == 4, 1u << kRowEmpty,
                        (int64_t)blockIdx.x * kWarpsPerBlock + w, (int64_t)gridDim.x * kWarpsPerBlock, lane, pol);
     // the last warp out resets the queue counters for the next launch that
