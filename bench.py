@@ -41,6 +41,24 @@ def peaks():
         return 6650.0, "fallback"
 
 
+# measured gather ceiling for the bench workload's own column sequence
+# (tools/gather_replay.cu, profiles/r1_gather_replay.md): pure 512-B B-row
+# gathers at the best depth (U = 8, 4 blocks/SM), CSR order
+GATHER_CEILING = {"c2_rmat20": (20649.0, "profiles/r1_gather_replay.md: c2 column sequence replayed as pure "
+                                         "512-B row gathers, U=8, 4 blocks/SM, 0.399 ms")}
+
+
+def gather_roofline(config, nnz, J, world, spmm_ms):
+    """The SpMM's binding traffic: one J*4-byte B row per nonzero through
+    L2/L1 (nnz*J*4 bytes per launch), against the measured gather ceiling."""
+    g = nnz * J * 4 / world
+    out = {"bytes_per_launch": int(g), "achieved": g / (spmm_ms * 1e-3) / 1e9, "unit": "GB/s"}
+    if config in GATHER_CEILING and world == 1:
+        c, src = GATHER_CEILING[config]
+        out.update(ceiling=c, frac=out["achieved"] / c, ceiling_source=src)
+    return out
+
+
 def algorithmic_bytes(A_h, J):
     """bytes_alg = nnz*(4+4) + U*J*4 + I*J*4: index + value of
     every nonzero once, each needed B row once, every C row written once."""
@@ -224,7 +242,10 @@ def main():
     d_rp, d_ci, d_va, d_B = (t.to(dev) for t in (h_rp, h_ci, h_va, h_B))
     A = lf.Csr(d_rp, d_ci, d_va, A_h.n_cols, p1 - p0)
     I_loc = hi - lo
-    C_loc = torch.empty((I_loc, J), dtype=torch.float32, device=dev)
+    # N > 1: every rank holds the full C; its SpMM writes its own rows in place
+    # and exchange_rows (NCCL point-to-point, exact sizes) fills in the rest
+    C_full = torch.empty((A_h.n_rows, J), dtype=torch.float32, device=dev) if world > 1 else None
+    C_loc = C_full[lo:hi] if world > 1 else torch.empty((I_loc, J), dtype=torch.float32, device=dev)
     h_C = torch.empty((I_loc, J), dtype=torch.float32).pin_memory()
     stream = torch.cuda.current_stream()
     kw = {}
@@ -246,7 +267,7 @@ def main():
         M.spmm(d_B, out=C_loc)
         e3 = ev(); e3.record(stream)
         if world > 1:
-            lfd.gather_rows(C_loc, bounds)
+            lfd.exchange_rows(C_full, bounds)
         e4 = ev(); e4.record(stream)
         if record:
             phase["_ev"].append((e0, e1, e2, e3, e4))
@@ -323,7 +344,7 @@ def main():
             Mi = lf.CellMatrix.build(Ain, pr, sti)
             Mi.spmm(d_B, out=C_loc)
             if world > 1:
-                lfd.gather_rows(C_loc, bounds)
+                lfd.exchange_rows(C_full, bounds)
             h_C.copy_(C_loc, non_blocking=True)
             Mi.close()
 
@@ -347,7 +368,13 @@ def main():
         return 0
     hbm_peak, peak_kind = peaks()
     P = params.n_parts
-    launches_per_step = 2 + (4 + (1 if P > 1 else 0)) + 2
+    # configure: features_kernel + stats_rows/mark/cols; build: bucket_kernel<0>,
+    # tile_scan, bucket_kernel<1>, slot_fill, run_bounds (+ seg_kernel for P > 1);
+    # SpMM: zero_rows_kernel + cell_spmm_kernel (CSR format: csr_spmm_kernel only)
+    if params.use_cell:
+        launches_per_step = 4 + 5 + (1 if P > 1 else 0) + 2
+    else:
+        launches_per_step = 4 + 1
     sp_ms = ph["spmm"]
     line = {
         "metric": METRIC, "value": flops / (ms * 1e-3) / 1e9, "unit": "GFLOP/s", "n_gpus": world,
@@ -365,6 +392,7 @@ def main():
                      "achieved": bytes_alg / world / (sp_ms * 1e-3) / 1e9, "peak": hbm_peak, "unit": "GB/s",
                      "frac": bytes_alg / world / (sp_ms * 1e-3) / 1e9 / hbm_peak, "peak_kind": peak_kind,
                      "bytes_alg_per_launch": bytes_alg // world, "traffic": None},
+        "gather": gather_roofline(args.config, A_h.nnz, J, world, sp_ms),
         "clocks": clk.summary(),
         "gpu_launches": launches_per_step * args.steps,
         "e2e": e2e,

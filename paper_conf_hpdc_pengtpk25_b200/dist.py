@@ -40,25 +40,72 @@ def shard_bounds(row_ptr: np.ndarray, world: int, J: int = 0, mode: str = "nnz")
     return b
 
 
+def exchange_rows(C: torch.Tensor, bounds, group=None) -> torch.Tensor:
+    """In place: C is the full [I, J] result on every rank, whose rows
+    [bounds[rank], bounds[rank+1]) this rank computed.  Every rank sends its
+    block to every peer and receives theirs straight into their rows (one
+    batched set of point-to-point transfers, exact sizes: no padding and no
+    staging copy; NCCL over NVLink/NVSwitch on GPUs)."""
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    if world == 1:
+        return C
+    b = [int(x) for x in bounds]
+    mine = C[b[rank]:b[rank + 1]]
+    ops = []
+    for r in range(world):
+        if r == rank:
+            continue
+        peer = dist.get_global_rank(group, r) if group is not None else r
+        if b[rank + 1] > b[rank]:
+            ops.append(dist.P2POp(dist.isend, mine, peer, group))
+        if b[r + 1] > b[r]:
+            ops.append(dist.P2POp(dist.irecv, C[b[r]:b[r + 1]], peer, group))
+    if ops:
+        for req in dist.batch_isend_irecv(ops):
+            req.wait()
+    return C
+
+
 def gather_rows(C_local: torch.Tensor, bounds, group=None) -> torch.Tensor:
-    """All-gather the ranks' row blocks of C into the full [I, J] matrix.
-    Shards are padded to the largest shard so a single all_gather_into_tensor
-    (NCCL) moves them; the padding is dropped on unpacking."""
+    """All-gather the ranks' row blocks of C into a new full [I, J] matrix
+    (exchange_rows after placing the local block)."""
+    rank = dist.get_rank(group)
+    b = [int(x) for x in bounds]
+    C = torch.empty((b[-1], C_local.shape[1]), dtype=C_local.dtype, device=C_local.device)
+    C[b[rank]:b[rank + 1]] = C_local
+    return exchange_rows(C, bounds, group)
+
+
+def col_bounds(J: int, world: int, align: int = 4) -> np.ndarray:
+    """world+1 column boundaries of B / C for the large-J mode:
+    near-equal slabs, every inner boundary a multiple of `align` (so each
+    slab keeps the 16-byte vector path of lf_spmm when J % 4 == 0)."""
+    units = -(-int(J) // align)
+    b = np.array([min(int(J), ((r * units) // world) * align) for r in range(world + 1)], np.int64)
+    b[world] = int(J)
+    return b
+
+
+def gather_cols(C_slab: torch.Tensor, cbounds, group=None) -> torch.Tensor:
+    """All-gather column slabs [I, J_r] into the full [I, J] C (one
+    all_gather of the padded slabs, then one strided copy per slab)."""
     world = dist.get_world_size(group)
-    sizes = np.diff(np.asarray(bounds, np.int64))
-    rmax = int(sizes.max()) if len(sizes) else 0
-    J = C_local.shape[1]
-    pad = torch.zeros((rmax, J), dtype=C_local.dtype, device=C_local.device)
-    pad[:C_local.shape[0]] = C_local
+    cb = [int(x) for x in cbounds]
+    wmax = max(cb[r + 1] - cb[r] for r in range(world))
+    I = C_slab.shape[0]
+    pad = torch.zeros((I, wmax), dtype=C_slab.dtype, device=C_slab.device)
+    pad[:, :C_slab.shape[1]] = C_slab
     if dist.get_backend(group) == "nccl":
-        buf = torch.empty((world * rmax, J), dtype=C_local.dtype, device=C_local.device)
+        buf = torch.empty((world, I, wmax), dtype=C_slab.dtype, device=C_slab.device)
         dist.all_gather_into_tensor(buf, pad, group=group)
-        parts = [buf[r * rmax: r * rmax + int(sizes[r])] for r in range(world)]
+        parts = [buf[r] for r in range(world)]
     else:
-        bufs = [torch.empty_like(pad) for _ in range(world)]
-        dist.all_gather(bufs, pad, group=group)
-        parts = [bufs[r][:int(sizes[r])] for r in range(world)]
-    return torch.cat(parts, dim=0)
+        parts = [torch.empty_like(pad) for _ in range(world)]
+        dist.all_gather(parts, pad, group=group)
+    C = torch.empty((I, cb[-1]), dtype=C_slab.dtype, device=C_slab.device)
+    for r in range(world):
+        C[:, cb[r]:cb[r + 1]] = parts[r][:, :cb[r + 1] - cb[r]]
+    return C
 
 
 def broadcast_B(B: torch.Tensor, src: int = 0, group=None) -> torch.Tensor:
@@ -70,7 +117,8 @@ def spmm_rowsharded(A_full, B: torch.Tensor, J: int, group=None, mode: str = "nn
                     **configure_kw):
     """C = A . B with A's rows sharded over the group.  A_full is this rank's
     handle on the whole CSR (lf.Csr on the local GPU); returns the full C (or
-    the local block when gather=False) and the bounds."""
+    the local block when gather=False) and the bounds.  The local SpMM writes
+    straight into its rows of the full C, which exchange_rows completes."""
     from . import CellMatrix, Csr, configure
     rank, world = dist.get_rank(group), dist.get_world_size(group)
     rp_host = A_full.row_ptr.cpu().numpy()
@@ -80,7 +128,27 @@ def spmm_rowsharded(A_full, B: torch.Tensor, J: int, group=None, mode: str = "nn
                 int(rp_host[hi] - rp_host[lo]))
     params, stats = configure(shard, J, **configure_kw)
     M = CellMatrix.build(shard, params, stats)
-    C_local = M.spmm(B)
     if not gather:
-        return C_local, bounds
-    return gather_rows(C_local, bounds, group), bounds
+        return M.spmm(B), bounds
+    C = torch.empty((A_full.n_rows, B.shape[1]), dtype=torch.float32, device=B.device)
+    M.spmm(B, out=C[lo:hi])
+    return exchange_rows(C, bounds, group), bounds
+
+
+def spmm_colsplit(A_full, B: torch.Tensor, group=None, gather: bool = True, **configure_kw):
+    """Large-J mode: every rank holds all of A (one CELL
+    handle) and multiplies its column slab of B, C[:, j0:j1] = A . B[:, j0:j1]
+    (lf_spmm on strided views: ldb = ldc = J, no slab copies of B).  Returns
+    the full C (or this rank's [I, j1-j0] slab when gather=False) and the
+    column bounds."""
+    from . import CellMatrix, configure
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    J = B.shape[1]
+    cb = col_bounds(J, world)
+    j0, j1 = int(cb[rank]), int(cb[rank + 1])
+    params, stats = configure(A_full, max(j1 - j0, 1), **configure_kw)
+    M = CellMatrix.build(A_full, params, stats)
+    C_slab = M.spmm(B[:, j0:j1])
+    if not gather:
+        return C_slab, cb
+    return gather_cols(C_slab, cb, group), cb

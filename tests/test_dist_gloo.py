@@ -37,7 +37,14 @@ def _worker(rank, world, port, mode, q):
         C_loc, _ = oracle.spmm_csr(A, B, rows=np.arange(lo, hi, dtype=np.int64), with_abs=False)
         C = lfd.gather_rows(torch.from_numpy(C_loc.astype(np.float64)), bounds)
         full, _ = oracle.spmm_csr(A, B, with_abs=False)
-        q.put((rank, bool(np.array_equal(C.numpy(), full)), bounds.tolist()))
+        ok = bool(np.array_equal(C.numpy(), full))
+        # large-J mode: column slabs of B, each rank's slab of C, gathered
+        cb = lfd.col_bounds(J, world)
+        j0, j1 = int(cb[rank]), int(cb[rank + 1])
+        C_slab, _ = oracle.spmm_csr(A, np.ascontiguousarray(B[:, j0:j1]), with_abs=False)
+        Cc = lfd.gather_cols(torch.from_numpy(C_slab.astype(np.float64)), cb)
+        ok = ok and bool(np.array_equal(Cc.numpy(), full))
+        q.put((rank, ok, bounds.tolist()))
     finally:
         dist.destroy_process_group()
 
@@ -55,6 +62,17 @@ def test_rowsharded_gather_world2(mode):
         p.join(timeout=60)
     assert all(ok for _, ok, _ in res)
     assert res[0][2] == res[1][2]
+
+
+def test_col_bounds_properties():
+    from paper_conf_hpdc_pengtpk25_b200 import dist as lfd
+    for J in (1, 4, 30, 128, 256, 512, 1000):
+        for world in (1, 2, 3, 4, 8):
+            b = lfd.col_bounds(J, world)
+            assert b[0] == 0 and b[-1] == J and len(b) == world + 1 and np.all(np.diff(b) >= 0)
+            assert all(x % 4 == 0 for x in b[1:-1])
+            w = np.diff(b)
+            assert w.max() - w[w > 0].min() <= 4 if (w > 0).any() else True
 
 
 def test_shard_bounds_properties():
