@@ -48,6 +48,12 @@ GATHER_CEILING = {"c2_rmat20": (20649.0, "profiles/r1_gather_replay.md: c2 colum
                                          "512-B row gathers, U=8, 4 blocks/SM, 0.399 ms")}
 
 
+# DRAM bytes per lf_spmm launch (dram__bytes_read.sum + dram__bytes_write.sum
+# of cell_spmm_kernel, ncu --set full, profiles/r1_bench_summary.md)
+NCU_TRAFFIC = {"c2_rmat20": (1503361000 + 535485952, "ncu --set full of cell_spmm_kernel (round 1, r1d): "
+                                                      "1.503 GB read + 0.535 GB written")}
+
+
 def gather_roofline(config, nnz, J, world, spmm_ms):
     """The SpMM's binding traffic: one J*4-byte B row per nonzero through
     L2/L1 (nnz*J*4 bytes per launch), against the measured gather ceiling."""
@@ -391,7 +397,10 @@ def main():
         "roofline": {"kernel": "lf_spmm (zero_rows + cell_spmm_kernel)", "bound": "hbm",
                      "achieved": bytes_alg / world / (sp_ms * 1e-3) / 1e9, "peak": hbm_peak, "unit": "GB/s",
                      "frac": bytes_alg / world / (sp_ms * 1e-3) / 1e9 / hbm_peak, "peak_kind": peak_kind,
-                     "bytes_alg_per_launch": bytes_alg // world, "traffic": None},
+                     "bytes_alg_per_launch": bytes_alg // world,
+                     "traffic": NCU_TRAFFIC[args.config][0] if args.config in NCU_TRAFFIC and world == 1 else None,
+                     "traffic_source": NCU_TRAFFIC[args.config][1] if args.config in NCU_TRAFFIC and world == 1
+                     else None},
         "gather": gather_roofline(args.config, A_h.nnz, J, world, sp_ms),
         "clocks": clk.summary(),
         "gpu_launches": launches_per_step * args.steps,

@@ -310,3 +310,28 @@ def test_repeated_launches_reuse_counter_slots(lf):
     torch.cuda.synchronize()
     for C in outs[::7] + outs[-3:]:
         assert np.array_equal(C.cpu().numpy().astype(np.float64), ref)
+
+
+def test_host_pipeline_overlapped(lf):
+    """HostPipeline: host CSR + B in, host C out, double-buffered over three
+    streams; several different problems in flight give their own results."""
+    from paper_conf_hpdc_pengtpk25_b200.pipeline import HostPipeline
+    J = 64
+    probs = []
+    for seed in range(4):
+        A_h = gen.rmat(11, 8 + 4 * seed, seed=seed, kind=gen.INT)
+        B_h = gen.dense(A_h.n_cols, J, seed, gen.INT)
+        probs.append((A_h, B_h))
+    I, K = probs[0][0].n_rows, probs[0][0].n_cols
+    pipe = HostPipeline(I, K, max(a.nnz for a, _ in probs), J)
+    outs = []
+    for it in range(8):
+        A_h, B_h = probs[it % 4]
+        h = [torch.from_numpy(x).pin_memory() for x in (A_h.row_ptr, A_h.col_ind, A_h.val, B_h)]
+        hC = torch.empty((I, J), dtype=torch.float32).pin_memory()
+        pipe.submit(*h, hC)
+        outs.append((it % 4, hC))
+    pipe.synchronize()
+    for i, hC in outs:
+        A_h, B_h = probs[i]
+        assert np.array_equal(hC.numpy().astype(np.float64), oracle.spmm_csr(A_h, B_h)[0])
