@@ -342,30 +342,25 @@ def main():
         h2d = sum(t.numel() * t.element_size() for t in (h_rp, h_ci, h_va, h_B))
         d2h = h_C.numel() * 4
 
-        def e2e_step():
-            for hs, ds in ((h_rp, d_rp), (h_ci, d_ci), (h_va, d_va), (h_B, d_B)):
-                ds.copy_(hs, non_blocking=True)
-            Ain = lf.Csr(d_rp, d_ci, d_va, A_h.n_cols, p1 - p0)
-            pr, sti = lf.configure(Ain, J, **kw)
-            Mi = lf.CellMatrix.build(Ain, pr, sti)
-            Mi.spmm(d_B, out=C_loc)
-            if world > 1:
-                lfd.exchange_rows(C_full, bounds)
-            h_C.copy_(C_loc, non_blocking=True)
-            Mi.close()
-
-        for _ in range(2):
-            e2e_step()
-        torch.cuda.synchronize()
+        # the public host-buffer API: HostPipeline (paper_conf_hpdc_pengtpk25_b200/pipeline.py)
+        # double-buffers the problem over H2D / compute / D2H streams, so step k+1's
+        # inputs stream in while step k computes and step k-1's C streams out
+        from paper_conf_hpdc_pengtpk25_b200.pipeline import HostPipeline
+        pipe = HostPipeline(I_loc, A_h.n_cols, p1 - p0, J, dev, **kw)
+        h_Cs = [h_C, torch.empty_like(h_C).pin_memory()]
+        for i in range(2):
+            pipe.submit(h_rp, h_ci, h_va, h_B, h_Cs[i % 2])
+        pipe.synchronize()
         x0, x1 = ev(), ev()
-        x0.record(stream)
         n_e2e = max(3, min(args.steps, 20))
-        for _ in range(n_e2e):
-            e2e_step()
-        x1.record(stream)
-        torch.cuda.synchronize()
+        x0.record(pipe.s_h2d)
+        for i in range(n_e2e):
+            pipe.submit(h_rp, h_ci, h_va, h_B, h_Cs[i % 2])
+        x1.record(pipe.s_d2h)
+        pipe.synchronize()
         e2e_ms = maxr(x0.elapsed_time(x1) / n_e2e)
         e2e = {"value": flops / (e2e_ms * 1e-3) / 1e9, "unit": "GFLOP/s", "ms_per_step": e2e_ms,
+               "api": "HostPipeline.submit (host CSR + B in, host C out; N > 1: each rank's row block)",
                "h2d_bytes_per_step": int(h2d * world), "d2h_bytes_per_step": int(d2h * world)}
 
     if rank != 0:

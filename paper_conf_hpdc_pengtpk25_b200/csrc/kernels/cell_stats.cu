@@ -38,6 +38,39 @@ __device__ __forceinline__ unsigned long long warp_sum_u31(unsigned v) {
     return ((unsigned long long)hi << 16) + lo;
 }
 
+// Block reduction of the four row-length statistics, then one set of 64-bit
+// atomics per block (per-warp atomics on the same four words serialise).
+__device__ __forceinline__ void block_len_stats(unsigned long long mn, unsigned long long mx, unsigned long long sum,
+                                                unsigned long long sq, StatsDev *st) {
+    __shared__ unsigned long long red[4][kThreads / 32];
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    for (int o = 16; o; o >>= 1) {
+        mn = min(mn, __shfl_xor_sync(kFull, mn, o));
+        mx = max(mx, __shfl_xor_sync(kFull, mx, o));
+        sum += __shfl_xor_sync(kFull, sum, o);
+        sq += __shfl_xor_sync(kFull, sq, o);
+    }
+    if (lane == 0) {
+        red[0][warp] = mn;
+        red[1][warp] = mx;
+        red[2][warp] = sum;
+        red[3][warp] = sq;
+    }
+    __syncthreads();
+    if (threadIdx.x == 0) {
+        for (int w = 1; w < (int)(blockDim.x >> 5); w++) {
+            mn = min(mn, red[0][w]);
+            mx = max(mx, red[1][w]);
+            sum += red[2][w];
+            sq += red[3][w];
+        }
+        atomicMin(&st->len_min, mn);
+        atomicMax(&st->len_max, mx);
+        atomicAdd(&st->len_sum, sum);
+        atomicAdd(&st->len_sumsq, sq);
+    }
+}
+
 // Pass 1 -- one thread per row: segments of the row in every partition, their
 // natural bucket t0 (written to t0seg[i*P+p]), the H / F histograms
 // (warp-aggregated: __match_any_sync for H, REDUX for F) and the Table 2
@@ -108,19 +141,7 @@ __global__ void __launch_bounds__(kThreads) stats_rows_kernel(const int64_t *__r
             b = e;
         }
     }
-    for (int o = 16; o; o >>= 1) {
-        mn = min(mn, __shfl_xor_sync(kFull, mn, o));
-        mx = max(mx, __shfl_xor_sync(kFull, mx, o));
-        sum += __shfl_xor_sync(kFull, sum, o);
-        sq += __shfl_xor_sync(kFull, sq, o);
-    }
-    if (lane == 0) {
-        atomicMin(&st->len_min, mn);
-        atomicMax(&st->len_max, mx);
-        atomicAdd(&st->len_sum, sum);
-        atomicAdd(&st->len_sumsq, sq);
-    }
-    __syncthreads();
+    block_len_stats(mn, mx, sum, sq, st);  // its __syncthreads also orders the H_s / F_s updates
     for (int q = threadIdx.x; q < P * kMaxT; q += blockDim.x) {
         if (H_s[q]) atomicAdd(&st->part[q / kMaxT].H[q % kMaxT], H_s[q]);
         if (F_s[q]) atomicAdd(&st->part[q / kMaxT].F[q % kMaxT], F_s[q]);
@@ -309,7 +330,6 @@ namespace {
 // 64-bit atomics per warp.
 __global__ void __launch_bounds__(kThreads) features_kernel(const int64_t *__restrict__ row_ptr, int64_t n_rows,
                                                             StatsDev *st) {
-    const int lane = threadIdx.x & 31;
     unsigned long long mn = ~0ull, mx = 0, sum = 0, sq = 0;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_rows; i += stride) {
@@ -319,18 +339,7 @@ __global__ void __launch_bounds__(kThreads) features_kernel(const int64_t *__res
         sum += len;
         sq += len * len;
     }
-    for (int o = 16; o; o >>= 1) {
-        mn = min(mn, __shfl_xor_sync(kFull, mn, o));
-        mx = max(mx, __shfl_xor_sync(kFull, mx, o));
-        sum += __shfl_xor_sync(kFull, sum, o);
-        sq += __shfl_xor_sync(kFull, sq, o);
-    }
-    if (lane == 0) {
-        atomicMin(&st->len_min, mn);
-        atomicMax(&st->len_max, mx);
-        atomicAdd(&st->len_sum, sum);
-        atomicAdd(&st->len_sumsq, sq);
-    }
+    block_len_stats(mn, mx, sum, sq, st);
 }
 
 }  // namespace
