@@ -61,7 +61,7 @@ __device__ __forceinline__ void segment_of(const int64_t *__restrict__ row_ptr, 
 template <int PASS>
 __global__ void __launch_bounds__(kThreads)
     bucket_kernel(const int64_t *__restrict__ row_ptr, const int32_t *__restrict__ seg_rel, int64_t n_rows, int P,
-                  const int8_t *__restrict__ e_of_p, int n_tiles, long long *__restrict__ tile_cnt,
+                  const __grid_constant__ WidthArg e_of_p, int n_tiles, long long *__restrict__ tile_cnt,
                   const long long *__restrict__ key_row_off, int32_t *__restrict__ row_cnt,
                   int32_t *__restrict__ row_ind, int32_t *__restrict__ row_tag, int64_t *__restrict__ src_pos,
                   int32_t *__restrict__ src_cnt, uint8_t *__restrict__ row_mode) {
@@ -69,7 +69,7 @@ __global__ void __launch_bounds__(kThreads)
     const int tile = blockIdx.x, p = blockIdx.y;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int64_t i = (int64_t)tile * kThreads + threadIdx.x;
-    const int e = e_of_p[p];
+    const int e = e_of_p.e[p];
 
     int64_t beg = 0, end = 0;
     if (i < n_rows) segment_of(row_ptr, seg_rel, i, p, P, beg, end);
@@ -105,9 +105,10 @@ __global__ void __launch_bounds__(kThreads)
     __syncthreads();
 
     if (PASS == 0) {
-        if (n_sub > 0) {
-            if (P == 1) row_cnt[i] = (int32_t)n_sub;
-            else atomicAdd(row_cnt + i, (int32_t)n_sub);
+        if (P == 1) {  // every entry written: no memset
+            if (i < n_rows) row_cnt[i] = (int32_t)n_sub;
+        } else if (n_sub > 0) {
+            atomicAdd(row_cnt + i, (int32_t)n_sub);
         }
         return;
     } else {
@@ -123,6 +124,8 @@ __global__ void __launch_bounds__(kThreads)
             const bool whole = row_cnt[i] == n_sub && key <= kPieceLog2 && (n_sub == 1 || (key >= 5 && n_sub <= kMaxRun));
             tag = (int32_t)((i << 3) | (whole ? 4 : 0));
             row_mode[i] = whole ? (n_sub == 1 ? kRowPlain : kRowRun) : kRowRed;
+        } else if (P == 1 && i < n_rows) {
+            row_mode[i] = kRowEmpty;  // (P > 1: pre-filled, another partition may own the row)
         }
         const int64_t W = int64_t(1) << (key == kNoKey ? 0 : key);
         if (n_sub <= 32) {
@@ -192,14 +195,43 @@ __global__ void __launch_bounds__(1024) tile_scan_kernel(long long *__restrict__
     if (threadIdx.x == 0) key_total[blockIdx.x] = carry;
 }
 
-constexpr int kSlotThreads = 256;
-constexpr int kSlotILP = 4;  // independent slots per thread per iteration
-constexpr int kMaxSmemBuckets = 2048;
+// one block per bucket: its block-padding rows, and (block 0) the counters
+__global__ void pad_init_kernel(const BucketDev *__restrict__ bk, int nb, int32_t *__restrict__ row_ind,
+                                int32_t *__restrict__ row_tag, int32_t *__restrict__ src_cnt,
+                                unsigned long long *__restrict__ ctr, int n_ctr) {
+    if (blockIdx.x == 0)
+        for (int q = threadIdx.x; q < n_ctr; q += blockDim.x) ctr[q] = 0;
+    if ((int)blockIdx.x >= nb) return;
+    const BucketDev b = bk[blockIdx.x];
+    for (int64_t r = b.row_off + b.n_real_rows + threadIdx.x; r < b.row_off + b.n_rows_pad; r += blockDim.x) {
+        row_ind[r] = -1;
+        row_tag[r] = -1;
+        src_cnt[r] = 0;
+    }
+}
 
-// One thread per slot (kSlotILP slots in flight per thread): bucket of the
-// slot (binary search over the bucket slot offsets in shared memory), its
-// CELL row and position w in the row; real slots copy colInd/val from the
-// CSR position src_pos[row] + w, the rest get the padding (-1, +0.0f).
+constexpr int kSlotThreads = 256;
+constexpr int kMaxSmemBuckets = 2048;
+constexpr int kSlotsPerLane = 4;                    // consecutive slots: one 16-byte store each
+constexpr int kSlotsPerWarp = 32 * kSlotsPerLane;   // a warp's chunk
+
+// A warp fills 128 consecutive slots per chunk, 4 per lane (vector stores).
+// The bucket of the chunk is found once (warp-uniform binary search over the
+// bucket slot offsets in shared memory); a chunk that straddles buckets
+// falls back to a per-slot search.  Slot s of bucket b is position
+// w = (s - soff) mod W of CELL row r = roff + (s - soff) / W; it copies
+// colInd / val from CSR position src_pos[r] + w when w < src_cnt[r]
+// (0 for block-padding rows), else the padding (-1, +0.0f).
+__device__ __forceinline__ int bucket_of(const int64_t *soff, int nb, int64_t s) {
+    int lo = 0, hi = nb - 1;  // last bucket with soff <= s
+    while (lo < hi) {
+        const int mid = (lo + hi + 1) >> 1;
+        if (soff[mid] <= s) lo = mid;
+        else hi = mid - 1;
+    }
+    return lo;
+}
+
 __global__ void __launch_bounds__(kSlotThreads)
     slot_fill_kernel(const int32_t *__restrict__ col, const float *__restrict__ val,
                      const BucketDev *__restrict__ bk, int nb, int64_t n_slots, const int64_t *__restrict__ src_pos,
@@ -214,46 +246,49 @@ __global__ void __launch_bounds__(kSlotThreads)
         tt[q] = bk[q].t;
     }
     __syncthreads();
-    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t s0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; s0 < n_slots; s0 += stride * kSlotILP) {
-        int64_t pos[kSlotILP];
-        int32_t cnt[kSlotILP], w[kSlotILP];
+    const int lane = threadIdx.x & 31;
+    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
+    for (int64_t ch = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; ch * kSlotsPerWarp < n_slots; ch += nw) {
+        const int64_t c0 = ch * kSlotsPerWarp;
+        const int bu = bucket_of(soff, nb, c0);  // uniform
+        const bool one = bu + 1 >= nb || soff[bu + 1] >= c0 + kSlotsPerWarp;
+        const int64_t s0 = c0 + lane * kSlotsPerLane;
+        int32_t c[kSlotsPerLane];
+        float v[kSlotsPerLane];
+        int64_t pos[kSlotsPerLane];
+        int32_t cnt[kSlotsPerLane], w[kSlotsPerLane];
 #pragma unroll
-        for (int k = 0; k < kSlotILP; k++) {
-            const int64_t s = s0 + k * stride;
+        for (int k = 0; k < kSlotsPerLane; k++) {
+            const int64_t s = s0 + k;
             cnt[k] = 0;
             w[k] = 1;
             pos[k] = 0;
             if (s < n_slots) {
-                int lo = 0, hi = nb - 1;  // last bucket with soff <= s
-                while (lo < hi) {
-                    const int mid = (lo + hi + 1) >> 1;
-                    if (soff[mid] <= s) lo = mid;
-                    else hi = mid - 1;
-                }
-                const int t = tt[lo];
-                const int64_t rel = s - soff[lo];
-                const int64_t r = roff[lo] + (rel >> t);
+                const int b = one ? bu : bucket_of(soff, nb, s);
+                const int t = tt[b];
+                const int64_t rel = s - soff[b];
+                const int64_t r = roff[b] + (rel >> t);
                 w[k] = (int32_t)(rel & ((int64_t(1) << t) - 1));
                 cnt[k] = __ldg(src_cnt + r);
                 pos[k] = __ldg(src_pos + r);
             }
         }
-        int32_t c[kSlotILP];
-        float v[kSlotILP];
 #pragma unroll
-        for (int k = 0; k < kSlotILP; k++) {
+        for (int k = 0; k < kSlotsPerLane; k++) {
             const bool real = w[k] < cnt[k];
             c[k] = real ? __ldg(col + pos[k] + w[k]) : -1;
             v[k] = real ? __ldg(val + pos[k] + w[k]) : 0.0f;
         }
+        if (s0 + kSlotsPerLane <= n_slots) {
+            __stcs(reinterpret_cast<int4 *>(col_out + s0), make_int4(c[0], c[1], c[2], c[3]));
+            __stcs(reinterpret_cast<float4 *>(val_out + s0), make_float4(v[0], v[1], v[2], v[3]));
+        } else {
 #pragma unroll
-        for (int k = 0; k < kSlotILP; k++) {
-            const int64_t s = s0 + k * stride;
-            if (s < n_slots) {
-                __stcs(col_out + s, c[k]);
-                __stcs(val_out + s, v[k]);
-            }
+            for (int k = 0; k < kSlotsPerLane; k++)
+                if (s0 + k < n_slots) {
+                    __stcs(col_out + s0 + k, c[k]);
+                    __stcs(val_out + s0 + k, v[k]);
+                }
         }
     }
 }
@@ -317,7 +352,7 @@ cudaError_t launch_seg(const lf_csr &A, int P, int32_t *seg_rel, cudaStream_t s)
     return cudaGetLastError();
 }
 
-cudaError_t launch_bucket_count(const lf_csr &A, int P, const int8_t *e, const BuildScratch &sc, int32_t *row_cnt,
+cudaError_t launch_bucket_count(const lf_csr &A, int P, const WidthArg &e, const BuildScratch &sc, int32_t *row_cnt,
                                 cudaStream_t s) {
     if (A.n_rows == 0) return cudaSuccess;
     dim3 grid(sc.n_tiles, P);
@@ -331,7 +366,13 @@ cudaError_t launch_tile_scan(int P, const BuildScratch &sc, cudaStream_t s) {
     return cudaGetLastError();
 }
 
-cudaError_t launch_bucket_place(const lf_csr &A, int P, const int8_t *e, const BuildScratch &sc,
+cudaError_t launch_pad_init(const BucketDev *bk, int nb, int32_t *row_ind, int32_t *row_tag, int32_t *src_cnt,
+                            unsigned long long *ctr, int n_ctr, cudaStream_t s) {
+    pad_init_kernel<<<std::max(nb, 1), 256, 0, s>>>(bk, nb, row_ind, row_tag, src_cnt, ctr, n_ctr);
+    return cudaGetLastError();
+}
+
+cudaError_t launch_bucket_place(const lf_csr &A, int P, const WidthArg &e, const BuildScratch &sc,
                                 const int32_t *row_cnt, int32_t *row_ind, int32_t *row_tag, uint8_t *row_mode,
                                 cudaStream_t s) {
     if (A.n_rows == 0) return cudaSuccess;
@@ -346,7 +387,8 @@ cudaError_t launch_slot_fill(const lf_csr &A, const BucketDev *d_buckets, int nb
                              const BuildScratch &sc, int32_t *col_out, float *val_out, cudaStream_t s) {
     if (n_slots == 0) return cudaSuccess;
     if (nb > kMaxSmemBuckets) return cudaErrorInvalidValue;
-    slot_fill_kernel<<<grid_for((n_slots + kSlotILP - 1) / kSlotILP, kSlotThreads), kSlotThreads, 0, s>>>(
+    static_assert(kSlotsPerLane == 4, "vector stores");
+    slot_fill_kernel<<<grid_for((n_slots + kSlotsPerLane - 1) / kSlotsPerLane, kSlotThreads), kSlotThreads, 0, s>>>(
         A.col_ind, A.val, d_buckets, nb, n_slots, sc.src_pos, sc.src_cnt, col_out, val_out);
     return cudaGetLastError();
 }

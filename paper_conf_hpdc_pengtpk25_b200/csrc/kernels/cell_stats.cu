@@ -79,9 +79,6 @@ __device__ __forceinline__ void block_len_stats(unsigned long long mn, unsigned 
 #define LF_MARK_TILE 4096
 #endif
 constexpr int kMarkTile = LF_MARK_TILE;
-#ifndef LF_MARK_L1
-#define LF_MARK_L1 0
-#endif
 #ifndef LF_MARK_MATCH
 #define LF_MARK_MATCH 0
 #endif  // nonzeros per block of the marking pass
@@ -161,9 +158,21 @@ __global__ void __launch_bounds__(kThreads) stats_rows_kernel(const int64_t *__r
 // The mask word of column c lives at slot hslot(c) = (c * odd) mod 2^m, a
 // bijection on [0, 2^m), 2^m >= K: columns that are hot together on power-law
 // inputs (small indices, few set bits) land on different L2 lines and slices.
-__device__ __forceinline__ uint32_t hslot(int32_t c, uint32_t kmask) { return ((uint32_t)c * 0x9E3779B1u) & kmask; }
+#ifndef LF_MARK_HASH
+#define LF_MARK_HASH 1
+#endif
+#ifndef LF_MARK_MODE
+#define LF_MARK_MODE 1  // 0: L2 check then RED; 1: RED only (measured fastest, c2: 107 vs 120 us); 2: L1-cached check
+#endif
+constexpr uint32_t kHashOdd = LF_MARK_HASH ? 0x9E3779B1u : 1u;
+__device__ __forceinline__ uint32_t hslot(int32_t c, uint32_t kmask) { return ((uint32_t)c * kHashOdd) & kmask; }
+__device__ __forceinline__ uint32_t ld_ca(const uint32_t *p) {
+    uint32_t v;
+    asm volatile("ld.global.ca.u32 %0, [%1];" : "=r"(v) : "l"(p));
+    return v;
+}
 
-__global__ void __launch_bounds__(kThreads) stats_mark_kernel(const int64_t *__restrict__ row_ptr,
+__global__ void __launch_bounds__(kThreads, 4) stats_mark_kernel(const int64_t *__restrict__ row_ptr,
                                                               const int32_t *__restrict__ col, int64_t n_rows,
                                                               int64_t S, int P,
                                                               const uint8_t *__restrict__ t0seg,
@@ -240,10 +249,9 @@ __global__ void __launch_bounds__(kThreads) stats_mark_kernel(const int64_t *__r
         if (P == 1) bit[k] = 1u << rt0[rr];
         else bit[k] = 1u << __ldg(t0seg + (rlo + rr) * P + (int)(c[k] / S));
     }
-    // L2 atomics are expensive (a few tens of G/s chip-wide) and most
-    // (column, bit) pairs are already set, so: keep one lane per distinct
-    // (column, bit) of the warp (__match_any_sync), read every mask word with one unconditional
-    // batch of L2 loads, and issue a RED only for bits still missing.
+    // One RED per (column, bit) (LF_MARK_MODE 1).  Reading the mask word
+    // first and skipping bits already set (mode 0) issues as many L2
+    // requests and adds a dependent load: measured slower on B200.
     uint32_t h[K], have[K];
 #pragma unroll
     for (int k = 0; k < K; k++) {
@@ -256,46 +264,82 @@ __global__ void __launch_bounds__(kThreads) stats_mark_kernel(const int64_t *__r
         h[k] = c[k] >= 0 ? hslot(c[k], kmask) : 0u;
     }
 #pragma unroll
-    for (int k = 0; k < K; k++) have[k] = LF_MARK_L1 ? mask[h[k]] : __ldcg(mask + h[k]);
+    for (int k = 0; k < K; k++)
+        have[k] = LF_MARK_MODE == 1 ? 0u : LF_MARK_MODE == 2 ? ld_ca(mask + h[k]) : __ldcg(mask + h[k]);
 #pragma unroll
     for (int k = 0; k < K; k++)
         if ((have[k] & bit[k]) != bit[k]) atomicOr(mask + h[k], bit[k]);
 }
 
+// Pass 3 -- one thread per mask SLOT (coalesced loads; the column is the
+// inverse of the slot hash, c = s * odd^-1 mod 2^m): Unat[p][t] = #{c : bit t},
+// Utop[p][t] = #{c : highest bit >= t}, the latter as a suffix sum of the
+// histogram of highest bits.  Warp-aggregated into shared-memory histograms.
+__host__ __device__ constexpr uint32_t inv_odd(uint32_t a) {
+    uint32_t x = a;  // Newton: x <- x (2 - a x), 5 steps give 32 bits
+    for (int i = 0; i < 5; i++) x *= 2u - a * x;
+    return x;
+}
+static_assert(kHashOdd * inv_odd(kHashOdd) == 1u, "hash inverse");
+
 __global__ void __launch_bounds__(kThreads) stats_cols_kernel(const uint32_t *__restrict__ mask, int64_t n_cols,
                                                               int64_t S, int P, StatsDev *st, uint32_t kmask) {
-    extern __shared__ unsigned long long sh[];  // Un_s[P][32], Ut_s[P][32]
-    unsigned long long *Un_s = sh, *Ut_s = sh + P * kMaxT;
+    extern __shared__ unsigned long long sh[];  // Un_s[P][32], Hb_s[P][32]
+    unsigned long long *Un_s = sh, *Hb_s = sh + P * kMaxT;
     for (int q = threadIdx.x; q < 2 * P * kMaxT; q += blockDim.x) sh[q] = 0;
     __syncthreads();
     const int lane = threadIdx.x & 31;
+    int cur_p = -1;
+    unsigned long long my_un = 0, my_hb = 0;
+    auto flush = [&]() {
+        if (cur_p >= 0 && lane < kMaxT) {
+            if (my_un) atomicAdd(&Un_s[cur_p * kMaxT + lane], my_un);
+            if (my_hb) atomicAdd(&Hb_s[cur_p * kMaxT + lane], my_hb);
+        }
+        my_un = my_hb = 0;
+    };
+    const int64_t n_slots = (int64_t)kmask + 1;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < n_cols; base += stride) {
-        const int64_t c = base + threadIdx.x;
-        const uint32_t m = c < n_cols ? __ldg(mask + hslot((int32_t)c, kmask)) : 0u;
-        const int p = c < n_cols ? (int)(c / S) : -1;
+    for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < n_slots; base += stride) {
+        const int64_t q = base + threadIdx.x;
+        uint32_t m = q < n_slots ? __ldcs(mask + q) : 0u;
+        const int64_t c = (int64_t)(((uint32_t)q * inv_odd(kHashOdd)) & kmask);
+        if (c >= n_cols) m = 0u;  // (a slot of no column holds 0 anyway)
+        const int p = m ? (int)(c / S) : -1;
         const int hb = m ? 31 - __clz(m) : -1;
-        // columns of one warp may straddle a partition boundary: group by p
+        // columns of one warp may lie in several partitions: group by p.
+        // Lane t counts bit t (Unat) and highest bit t (Hb) of the group's
+        // columns in registers; they go to shared memory when the partition
+        // changes (P = 1: once, after the loop)
         unsigned todo = __ballot_sync(kFull, m != 0);
         while (todo) {
             const int pp = __shfl_sync(kFull, p, __ffs(todo) - 1);
             const bool mine = m != 0 && p == pp;
             todo &= ~__ballot_sync(kFull, mine);
-            const int tmax = __reduce_max_sync(kFull, mine ? (unsigned)hb : 0u);
-            for (int t = 0; t <= tmax; t++) {
-                const unsigned un = __reduce_add_sync(kFull, mine && ((m >> t) & 1u));
-                const unsigned ut = __reduce_add_sync(kFull, mine && hb >= t);
-                if (lane == 0) {
-                    if (un) atomicAdd(&Un_s[pp * kMaxT + t], (unsigned long long)un);
-                    if (ut) atomicAdd(&Ut_s[pp * kMaxT + t], (unsigned long long)ut);
+            if (pp != cur_p) {
+                flush();
+                cur_p = pp;
+            }
+            const uint32_t mm = mine ? m : 0u;
+#pragma unroll
+            for (int t = 0; t < 32; t++) {
+                const unsigned un = __popc(__ballot_sync(kFull, (mm >> t) & 1u));
+                const unsigned nh = __popc(__ballot_sync(kFull, mine && hb == t));
+                if (lane == t) {
+                    my_un += un;
+                    my_hb += nh;
                 }
             }
         }
     }
+    flush();
     __syncthreads();
     for (int q = threadIdx.x; q < P * kMaxT; q += blockDim.x) {
-        if (Un_s[q]) atomicAdd(&st->part[q / kMaxT].Unat[q % kMaxT], Un_s[q]);
-        if (Ut_s[q]) atomicAdd(&st->part[q / kMaxT].Utop[q % kMaxT], Ut_s[q]);
+        const int p = q / kMaxT, t = q % kMaxT;
+        unsigned long long top = 0;  // Utop[t] = sum_{h >= t} Hb[h]
+        for (int h = t; h < kMaxT; h++) top += Hb_s[p * kMaxT + h];
+        if (Un_s[q]) atomicAdd(&st->part[p].Unat[t], Un_s[q]);
+        if (top) atomicAdd(&st->part[p].Utop[t], top);
     }
 }
 
@@ -322,36 +366,6 @@ uint32_t mask_slots(int64_t n_cols) {
     return (uint32_t)m;
 }
 
-namespace {
-
-// Table 2 row-length statistics alone: the features the
-// predictor needs BEFORE P is known (section 5.1-5.2), from row_ptr only
-// (8 B per row).  One thread per row, warp then block reduction, one set of
-// 64-bit atomics per warp.
-__global__ void __launch_bounds__(kThreads) features_kernel(const int64_t *__restrict__ row_ptr, int64_t n_rows,
-                                                            StatsDev *st) {
-    unsigned long long mn = ~0ull, mx = 0, sum = 0, sq = 0;
-    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_rows; i += stride) {
-        const unsigned long long len = (unsigned long long)(__ldg(row_ptr + i + 1) - __ldg(row_ptr + i));
-        mn = min(mn, len);
-        mx = max(mx, len);
-        sum += len;
-        sq += len * len;
-    }
-    block_len_stats(mn, mx, sum, sq, st);
-}
-
-}  // namespace
-
-cudaError_t launch_features(const lf_csr &A, StatsDev *d_stats, cudaStream_t s) {
-    if (A.n_rows <= 0) return cudaSuccess;
-    const int64_t want = (A.n_rows + kThreads - 1) / kThreads;
-    const int grid = (int)std::min<int64_t>(want, (int64_t)num_sms() * 8);
-    features_kernel<<<grid, kThreads, 0, s>>>(A.row_ptr, A.n_rows, d_stats);
-    return cudaGetLastError();
-}
-
 cudaError_t launch_stats(const lf_csr &A, int P, StatsDev *d_stats, uint32_t *d_colmask, uint8_t *d_t0seg,
                          cudaStream_t s) {
     const int64_t S = A.n_cols > 0 ? (A.n_cols + P - 1) / P : 1;
@@ -371,7 +385,7 @@ cudaError_t launch_stats(const lf_csr &A, int P, StatsDev *d_stats, uint32_t *d_
                                                                     mask_slots(A.n_cols) - 1);
     }
     if (A.n_cols > 0) {
-        const int64_t want = (A.n_cols + kThreads - 1) / kThreads;
+        const int64_t want = ((int64_t)mask_slots(A.n_cols) + kThreads - 1) / kThreads;
         const int grid = (int)std::min<int64_t>(want, (int64_t)num_sms() * 8);
         stats_cols_kernel<<<grid, kThreads, hist, s>>>(d_colmask, A.n_cols, S, P, d_stats, mask_slots(A.n_cols) - 1);
     }

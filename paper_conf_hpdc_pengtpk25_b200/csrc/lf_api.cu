@@ -170,45 +170,45 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
     // pinned staging buffer (one per thread) so the copies back are plain DMAs
     thread_local lf::StatsDev *h_st = nullptr;
     if (!h_st) LF_CUDA(cudaMallocHost(&h_st, sizeof(lf::StatsDev)));
-    // predictor (sections 5.1-5.2): Table 2 features first, then format and P
-    int P = o.force_parts;
-    int use_cell = o.force_format == 2 ? 0 : 1;
-    if (o.force_parts == 0 || o.force_format == 0) {
-        lf::StatsDev *d_f = nullptr;
-        const size_t fb = lf::stats_bytes(0);
-        LF_CUDA(cudaMallocAsync(&d_f, fb, s));
-        LF_CUDA(cudaMemsetAsync(d_f, 0, fb, s));
-        LF_CUDA(cudaMemsetAsync(&d_f->len_min, 0xFF, sizeof(unsigned long long), s));
-        LF_CUDA(lf::launch_features(*A, d_f, s));
-        LF_CUDA(cudaMemcpyAsync(h_st, d_f, fb, cudaMemcpyDeviceToHost, s));
-        LF_CUDA(cudaFreeAsync(d_f, s));
+    // GPU statistics for P partitions (one scratch allocation: stats, column
+    // masks, per-segment t0 + mark tiles), copied back with one sync
+    auto run_stats = [&](int P) -> lf_status {
+        const size_t st_bytes = lf::stats_bytes(P);
+        const size_t words = A->n_cols > 0 ? lf::mask_slots(A->n_cols) : 0;
+        const size_t b_st = (st_bytes + 255) & ~size_t(255), b_mask = (words * 4 + 255) & ~size_t(255);
+        const size_t b_t0 = A->n_rows > 0 ? lf::stats_scratch_bytes(A->n_rows, A->nnz, P) : 0;
+        char *d = nullptr;
+        LF_CUDA(cudaMallocAsync(&d, b_st + b_mask + b_t0 + 256, s));
+        lf::StatsDev *d_st = reinterpret_cast<lf::StatsDev *>(d);
+        uint32_t *d_mask = words ? reinterpret_cast<uint32_t *>(d + b_st) : nullptr;
+        uint8_t *d_t0 = b_t0 ? reinterpret_cast<uint8_t *>(d + b_st + b_mask) : nullptr;
+        // stats and masks are adjacent: one memset zeroes both
+        LF_CUDA(cudaMemsetAsync(d, 0, b_st + b_mask, s));
+        LF_CUDA(cudaMemsetAsync(&d_st->len_min, 0xFF, sizeof(unsigned long long), s));
+        LF_CUDA(lf::launch_stats(*A, P, d_st, d_mask, d_t0, s));
+        LF_CUDA(cudaMemcpyAsync(h_st, d_st, st_bytes, cudaMemcpyDeviceToHost, s));
+        LF_CUDA(cudaFreeAsync(d, s));
         LF_CUDA(cudaStreamSynchronize(s));
+        return LF_OK;
+    };
+    // predictor (sections 5.1-5.2): it needs the Table 2 row-length features
+    // before P is known.  The statistics pass computes them too, so it runs
+    // once speculatively for P = 1 (the forced P if given) and only again if
+    // the predictor picks another P -- one pass and one sync in the common case.
+    int P = o.force_parts ? o.force_parts : 1;
+    int use_cell = o.force_format == 2 ? 0 : 1;
+    if (lf_status st = run_stats(P)) return st;
+    if (o.force_parts == 0 || o.force_format == 0) {
         double f[8];
         table2_features(*A, J, *h_st, f);
         int32_t pu = 1, pp = 1;
         if (lf_status st = lf_predict(f, max_parts, &pu, &pp)) return fail(st, "lf_predict");
         if (o.force_format == 0) use_cell = pu;
-        if (o.force_parts == 0) P = pp;
+        if (o.force_parts == 0 && pp != P) {
+            P = pp;
+            if (lf_status st = run_stats(P)) return st;
+        }
     }
-    lf::StatsDev *d_st = nullptr;
-    uint32_t *d_mask = nullptr;
-    const size_t st_bytes = lf::stats_bytes(P);
-    LF_CUDA(cudaMallocAsync(&d_st, st_bytes, s));
-    LF_CUDA(cudaMemsetAsync(d_st, 0, st_bytes, s));
-    LF_CUDA(cudaMemsetAsync(&d_st->len_min, 0xFF, sizeof(unsigned long long), s));
-    if (A->n_cols > 0) {
-        const size_t words = lf::mask_slots(A->n_cols);
-        LF_CUDA(cudaMallocAsync(&d_mask, words * sizeof(uint32_t), s));
-        LF_CUDA(cudaMemsetAsync(d_mask, 0, words * sizeof(uint32_t), s));
-    }
-    uint8_t *d_t0 = nullptr;
-    if (A->n_rows > 0) LF_CUDA(cudaMallocAsync(&d_t0, lf::stats_scratch_bytes(A->n_rows, A->nnz, P), s));
-    LF_CUDA(lf::launch_stats(*A, P, d_st, d_mask, d_t0, s));
-    LF_CUDA(cudaMemcpyAsync(h_st, d_st, st_bytes, cudaMemcpyDeviceToHost, s));
-    LF_CUDA(cudaFreeAsync(d_st, s));
-    if (d_mask) LF_CUDA(cudaFreeAsync(d_mask, s));
-    if (d_t0) LF_CUDA(cudaFreeAsync(d_t0, s));
-    LF_CUDA(cudaStreamSynchronize(s));
     const lf::StatsDev &st = *h_st;
 
     lf_configure_stats local;
@@ -294,37 +294,84 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
     Mem mem{al, s};
     const int64_t I = A->n_rows;
     const int n_tiles = (int)((I + lf::kBuildTile - 1) / lf::kBuildTile);
-    Scratch sc{mem, {}};
-    lf::BuildScratch bs{};
-    bs.n_tiles = n_tiles;
-    int8_t *d_e = sc.get<int8_t>(LF_MAX_PARTS);
-    bs.seg_rel = P > 1 ? sc.get<int32_t>((size_t)I * (P - 1)) : nullptr;
-    bs.tile_cnt = sc.get<long long>((size_t)P * lf::kMaxT * std::max(n_tiles, 1));
-    bs.key_total = sc.get<long long>((size_t)P * lf::kMaxT);
-    bs.key_row_off = sc.get<long long>((size_t)P * lf::kMaxT);
-    int32_t *row_cnt = sc.get<int32_t>((size_t)std::max<int64_t>(I, 1));
-    h->row_mode = static_cast<uint8_t *>(mem.get((size_t)std::max<int64_t>(I, 1)));
-    if (!d_e || !bs.tile_cnt || !bs.key_total || !bs.key_row_off || !row_cnt || !h->row_mode ||
-        (P > 1 && I > 0 && !bs.seg_rel))
-        return bail(fail(LF_ERR_NO_MEMORY, "scratch allocation failed"));
-
-    // a1 + a4 (count): segments, bucket keys, per-tile totals, tile scan
     auto cu = [&](cudaError_t e, const char *what) -> lf_status {
         if (e != cudaSuccess) return fail(LF_ERR_CUDA, std::string(what) + ": " + cudaGetErrorString(e));
         return LF_OK;
     };
     lf_status st;
-    if ((st = cu(cudaMemcpyAsync(d_e, params->max_width_log2, LF_MAX_PARTS, cudaMemcpyHostToDevice, s), "H2D e")))
-        return bail(st);
-    if ((st = cu(cudaMemsetAsync(row_cnt, 0, (size_t)std::max<int64_t>(I, 1) * sizeof(int32_t), s), "memset")))
-        return bail(st);
-    if ((st = cu(cudaMemsetAsync(h->row_mode, lf::kRowEmpty, (size_t)std::max<int64_t>(I, 1), s), "memset")))
-        return bail(st);
-    if ((st = cu(cudaMemsetAsync(bs.tile_cnt, 0, (size_t)P * lf::kMaxT * std::max(n_tiles, 1) * 8, s), "memset")))
-        return bail(st);
-    if ((st = cu(lf::launch_seg(*A, P, bs.seg_rel, s), "seg"))) return bail(st);
-    if ((st = cu(lf::launch_bucket_count(*A, P, d_e, bs, row_cnt, s), "bucket_count"))) return bail(st);
-    if (n_tiles > 0 && (st = cu(lf::launch_tile_scan(P, bs, s), "tile_scan"))) return bail(st);
+    lf::BuildScratch bs{};
+    bs.n_tiles = n_tiles;
+    lf::WidthArg e_arg{};
+    for (int p = 0; p < P; p++) e_arg.e[p] = params->max_width_log2[p];
+
+    // host: bucket table (R2, R7) and warp-task decomposition from the bucket
+    // sizes (CELL rows per (p, t))
+    int64_t R_tot = 0, S_tot = 0;
+    std::vector<long long> row_off((size_t)P * lf::kMaxT, -1);
+    auto make_table = [&](const std::vector<long long> &tot) -> lf_status {
+        std::vector<lf::BucketDev> bn, bw;
+        for (int p = 0; p < P; p++) {
+            const int k = params->block_nnz_log2[p];
+            for (int t = 0; t <= params->max_width_log2[p]; t++) {
+                const long long n = tot[(size_t)p * lf::kMaxT + t];
+                if (n == 0) continue;
+                const int64_t R = int64_t(1) << (k - t), W = int64_t(1) << t;
+                const int64_t pad = (n + R - 1) / R * R;
+                lf_bucket b{};
+                b.part = p;
+                b.width_log2 = t;
+                b.rows_per_block = (int32_t)std::min<int64_t>(R, INT32_MAX);
+                b.n_rows = n;
+                b.n_rows_pad = pad;
+                b.row_off = R_tot;
+                b.slot_off = S_tot;
+                h->buckets.push_back(b);
+                lf::BucketDev d{};
+                d.slot_off = S_tot;
+                d.row_off = R_tot;
+                d.n_slots = pad * W;
+                d.n_real_rows = n;
+                d.n_rows_pad = pad;
+                d.t = t;
+                d.piece_log2 = std::max(0, t - lf::kPieceLog2);
+                d.task_slots = (int32_t)std::max<int64_t>(32, W >> d.piece_log2);
+                if (W < 32) {
+                    d.task_off = h->n_tasks_n;
+                    h->n_tasks_n += (pad * W + 31) / 32;
+                    h->slots_n += pad * W;
+                    bn.push_back(d);
+                } else {
+                    d.task_off = h->n_tasks_w;
+                    h->n_tasks_w += pad << d.piece_log2;
+                    h->slots_w += pad * W;
+                    bw.push_back(d);
+                }
+                d.task_off = 0;
+                h->h_buckets.push_back(d);
+                row_off[(size_t)p * lf::kMaxT + t] = R_tot;
+                R_tot += pad;
+                S_tot += pad * W;
+            }
+        }
+        h->n_cell_rows = R_tot;
+        h->n_slots = S_tot;
+        h->nb_n = (int)bn.size();
+        h->nb_w = (int)bw.size();
+        h->h_buckets.insert(h->h_buckets.end(), bn.begin(), bn.end());
+        h->h_buckets.insert(h->h_buckets.end(), bw.begin(), bw.end());
+        if (h->buckets.size() > 2048) return fail(LF_ERR_UNSUPPORTED, "more than 2048 buckets");
+        return LF_OK;
+    };
+
+    // scratch, ONE allocation: [seg_rel | tile_cnt | key_total | row_cnt | src_pos | src_cnt]
+    // (src_* sized by R_tot: known up front when the configure stats are passed)
+    const size_t a256 = 256;
+    auto up = [&](size_t b) { return (b + a256 - 1) / a256 * a256; };
+    const size_t s_seg = P > 1 ? up((size_t)I * (P - 1) * 4) : 0,
+                 s_tc = up((size_t)P * lf::kMaxT * std::max(n_tiles, 1) * 8), s_kt = up((size_t)P * lf::kMaxT * 8),
+                 s_rc = up((size_t)std::max<int64_t>(I, 1) * 4);
+    const size_t s_head = s_seg + s_tc + s_kt + s_rc;
+    Scratch sc{mem, {}};
     std::vector<long long> tot((size_t)P * lf::kMaxT, 0);
     if (stats) {  // bucket sizes from the configure statistics: no synchronisation
         for (int p = 0; p < P; p++) {
@@ -332,109 +379,84 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
             for (int t = 0; t < e && t < lf::kMaxT; t++) tot[(size_t)p * lf::kMaxT + t] = stats->H[p][t];
             if (e < lf::kMaxT) tot[(size_t)p * lf::kMaxT + e] = stats->F[p][e];
         }
-    } else {
+        if ((st = make_table(tot))) return bail(st);
+    }
+    const size_t s_src = stats ? up((size_t)R_tot * 8) + up((size_t)R_tot * 4) : 0;
+    char *scr = sc.get<char>(s_head + s_src);
+    if (!scr) return bail(fail(LF_ERR_NO_MEMORY, "scratch allocation failed"));
+    bs.seg_rel = P > 1 ? reinterpret_cast<int32_t *>(scr) : nullptr;
+    bs.tile_cnt = reinterpret_cast<long long *>(scr + s_seg);
+    bs.key_total = reinterpret_cast<long long *>(scr + s_seg + s_tc);
+    int32_t *row_cnt = reinterpret_cast<int32_t *>(scr + s_seg + s_tc + s_kt);
+
+    // a1 + a4 (count): segments, bucket keys, per-tile totals, tile scan
+    // (P = 1: bucket_kernel<0> writes every row_cnt entry itself)
+    if (P > 1 && I > 0 &&
+        (st = cu(cudaMemsetAsync(row_cnt, 0, (size_t)I * sizeof(int32_t), s), "memset")))
+        return bail(st);
+    if ((st = cu(lf::launch_seg(*A, P, bs.seg_rel, s), "seg"))) return bail(st);
+    if ((st = cu(lf::launch_bucket_count(*A, P, e_arg, bs, row_cnt, s), "bucket_count"))) return bail(st);
+    if (n_tiles > 0 && (st = cu(lf::launch_tile_scan(P, bs, s), "tile_scan"))) return bail(st);
+    if (!stats) {
         if (n_tiles > 0 &&
             (st = cu(cudaMemcpyAsync(tot.data(), bs.key_total, tot.size() * 8, cudaMemcpyDeviceToHost, s), "D2H")))
             return bail(st);
         if ((st = cu(cudaStreamSynchronize(s), "sync"))) return bail(st);
+        if ((st = make_table(tot))) return bail(st);
+        char *src = sc.get<char>(up((size_t)R_tot * 8) + up((size_t)R_tot * 4));
+        if (R_tot && !src) return bail(fail(LF_ERR_NO_MEMORY, "scratch allocation failed"));
+        bs.src_pos = reinterpret_cast<int64_t *>(src);
+        bs.src_cnt = R_tot ? reinterpret_cast<int32_t *>(src + up((size_t)R_tot * 8)) : nullptr;
+    } else {
+        bs.src_pos = reinterpret_cast<int64_t *>(scr + s_head);
+        bs.src_cnt = reinterpret_cast<int32_t *>(scr + s_head + up((size_t)R_tot * 8));
     }
-
-    // host: bucket table (R2, R7) and warp-task decomposition
-    std::vector<long long> row_off((size_t)P * lf::kMaxT, -1);
-    int64_t R_tot = 0, S_tot = 0;
-    std::vector<lf::BucketDev> bn, bw;
-    for (int p = 0; p < P; p++) {
-        const int k = params->block_nnz_log2[p];
-        for (int t = 0; t <= params->max_width_log2[p]; t++) {
-            const long long n = tot[(size_t)p * lf::kMaxT + t];
-            if (n == 0) continue;
-            const int64_t R = int64_t(1) << (k - t), W = int64_t(1) << t;
-            const int64_t pad = (n + R - 1) / R * R;
-            lf_bucket b{};
-            b.part = p;
-            b.width_log2 = t;
-            b.rows_per_block = (int32_t)std::min<int64_t>(R, INT32_MAX);
-            b.n_rows = n;
-            b.n_rows_pad = pad;
-            b.row_off = R_tot;
-            b.slot_off = S_tot;
-            h->buckets.push_back(b);
-            lf::BucketDev d{};
-            d.slot_off = S_tot;
-            d.row_off = R_tot;
-            d.n_slots = pad * W;
-            d.t = t;
-            d.piece_log2 = std::max(0, t - lf::kPieceLog2);
-            d.task_slots = (int32_t)std::max<int64_t>(32, W >> d.piece_log2);
-            if (W < 32) {
-                d.task_off = h->n_tasks_n;
-                h->n_tasks_n += (pad * W + 31) / 32;
-                h->slots_n += pad * W;
-                bn.push_back(d);
-            } else {
-                d.task_off = h->n_tasks_w;
-                h->n_tasks_w += pad << d.piece_log2;
-                h->slots_w += pad * W;
-                bw.push_back(d);
-            }
-            d.task_off = 0;
-            h->h_buckets.push_back(d);
-            row_off[(size_t)p * lf::kMaxT + t] = R_tot;
-            R_tot += pad;
-            S_tot += pad * W;
-        }
-    }
-    h->n_cell_rows = R_tot;
-    h->n_slots = S_tot;
-    h->nb_n = (int)bn.size();
-    h->nb_w = (int)bw.size();
-    h->h_buckets.insert(h->h_buckets.end(), bn.begin(), bn.end());
-    h->h_buckets.insert(h->h_buckets.end(), bw.begin(), bw.end());
     const int nb = (int)h->buckets.size();
-    if (nb > 2048) return bail(fail(LF_ERR_UNSUPPORTED, "more than 2048 buckets"));
 
-    // persistent arrays: one pool
-    const size_t a256 = 256;
-    auto up = [&](size_t b) { return (b + a256 - 1) / a256 * a256; };
-    const size_t b_ri = up(R_tot * 4), b_rt = up(R_tot * 4), b_ci = up(S_tot * 4), b_va = up(S_tot * 4),
-                 b_bk = up(h->h_buckets.size() * sizeof(lf::BucketDev)),
-                 b_rb = up((size_t)(h->n_tasks_w + 1)), b_ct = up(kCtrSlots * 4 * sizeof(unsigned long long));
-    h->pool_bytes = b_ri + b_rt + b_ci + b_va + b_bk + b_rb + b_ct;
+    // persistent arrays, ONE allocation (the pool): a header copied with one
+    // H2D [bucket table | key_row_off], then rowInd, row tags, colInd, val,
+    // run bounds, queue counters, row modes
+    const size_t b_bk = up(h->h_buckets.size() * sizeof(lf::BucketDev)), b_ko = up(row_off.size() * 8),
+                 b_ri = up(R_tot * 4), b_rt = up(R_tot * 4), b_ci = up(S_tot * 4), b_va = up(S_tot * 4),
+                 b_rb = up((size_t)(h->n_tasks_w + 1)), b_ct = up(kCtrSlots * 4 * sizeof(unsigned long long)),
+                 b_rm = up((size_t)std::max<int64_t>(I, 1));
+    h->pool_bytes = b_bk + b_ko + b_ri + b_rt + b_ci + b_va + b_rb + b_ct + b_rm;
     h->pool = mem.get(h->pool_bytes);
-    if (h->pool_bytes && !h->pool) return bail(fail(LF_ERR_NO_MEMORY, "CELL arrays allocation failed"));
+    if (!h->pool) return bail(fail(LF_ERR_NO_MEMORY, "CELL arrays allocation failed"));
     char *q = static_cast<char *>(h->pool);
+    h->d_buckets = reinterpret_cast<lf::BucketDev *>(q);
+    bs.key_row_off = reinterpret_cast<long long *>(q + b_bk);
+    q += b_bk + b_ko;
     h->row_ind = reinterpret_cast<int32_t *>(q);
     h->row_tag = reinterpret_cast<int32_t *>(q + b_ri);
     h->col_ind = reinterpret_cast<int32_t *>(q + b_ri + b_rt);
     h->val = reinterpret_cast<float *>(q + b_ri + b_rt + b_ci);
-    h->d_buckets = reinterpret_cast<lf::BucketDev *>(q + b_ri + b_rt + b_ci + b_va);
-    h->run_bound = reinterpret_cast<uint8_t *>(q + b_ri + b_rt + b_ci + b_va + b_bk);
-    h->ctr_ring = reinterpret_cast<unsigned long long *>(q + b_ri + b_rt + b_ci + b_va + b_bk + b_rb);
-    if ((st = cu(cudaMemsetAsync(h->ctr_ring, 0, b_ct, s), "memset"))) return bail(st);
-    bs.src_pos = sc.get<int64_t>((size_t)R_tot);
-    bs.src_cnt = sc.get<int32_t>((size_t)R_tot);
-    if (R_tot && (!bs.src_pos || !bs.src_cnt)) return bail(fail(LF_ERR_NO_MEMORY, "scratch allocation failed"));
-
-    if (R_tot) {
-        if ((st = cu(cudaMemsetAsync(h->row_ind, 0xFF, R_tot * 4, s), "memset"))) return bail(st);
-        if ((st = cu(cudaMemsetAsync(h->row_tag, 0xFF, R_tot * 4, s), "memset"))) return bail(st);
-        if ((st = cu(cudaMemsetAsync(bs.src_cnt, 0, R_tot * 4, s), "memset"))) return bail(st);
+    h->run_bound = reinterpret_cast<uint8_t *>(q + b_ri + b_rt + b_ci + b_va);
+    h->ctr_ring = reinterpret_cast<unsigned long long *>(q + b_ri + b_rt + b_ci + b_va + b_rb);
+    h->row_mode = reinterpret_cast<uint8_t *>(q + b_ri + b_rt + b_ci + b_va + b_rb + b_ct);
+    {
+        std::vector<char> head(b_bk + b_ko, 0);
+        if (!h->h_buckets.empty())
+            std::memcpy(head.data(), h->h_buckets.data(), h->h_buckets.size() * sizeof(lf::BucketDev));
+        std::memcpy(head.data() + b_bk, row_off.data(), row_off.size() * 8);
+        if ((st = cu(cudaMemcpyAsync(h->pool, head.data(), head.size(), cudaMemcpyHostToDevice, s), "H2D table")))
+            return bail(st);
     }
-    if (nb && (st = cu(cudaMemcpyAsync(h->d_buckets, h->h_buckets.data(), h->h_buckets.size() * sizeof(lf::BucketDev),
-                                       cudaMemcpyHostToDevice, s),
-                       "H2D buckets")))
+    // P > 1: several blocks update one row's mode, so it starts at kRowEmpty
+    if (P > 1 && I > 0 && (st = cu(cudaMemsetAsync(h->row_mode, lf::kRowEmpty, (size_t)I, s), "memset")))
         return bail(st);
-    if ((st = cu(cudaMemcpyAsync(bs.key_row_off, row_off.data(), row_off.size() * 8, cudaMemcpyHostToDevice, s),
-                 "H2D row_off")))
+    // queue counters zero; padding rows' rowInd / tags -1 and src_cnt 0
+    if ((st = cu(lf::launch_pad_init(h->d_buckets, nb, h->row_ind, h->row_tag, bs.src_cnt, h->ctr_ring,
+                                     kCtrSlots * 4, s),
+                 "pad_init")))
         return bail(st);
     // a4 (place) + a5 (scatter)
-    if ((st = cu(lf::launch_bucket_place(*A, P, d_e, bs, row_cnt, h->row_ind, h->row_tag, h->row_mode, s),
+    if ((st = cu(lf::launch_bucket_place(*A, P, e_arg, bs, row_cnt, h->row_ind, h->row_tag, h->row_mode, s),
                  "bucket_place")))
         return bail(st);
     if ((st = cu(lf::launch_slot_fill(*A, h->d_buckets, nb, S_tot, bs, h->col_ind, h->val, s), "slot_fill")))
         return bail(st);
-    if (h->pool &&
-        (st = cu(lf::launch_run_bounds(h->d_buckets + nb + h->nb_n, h->nb_w, h->n_tasks_w, h->row_tag, h->run_bound,
+    if ((st = cu(lf::launch_run_bounds(h->d_buckets + nb + h->nb_n, h->nb_w, h->n_tasks_w, h->row_tag, h->run_bound,
                                        s),
                  "run_bounds")))
         return bail(st);
@@ -497,7 +519,6 @@ lf_status lf_cell_destroy(lf_cell *h) {
     if (!h) return LF_OK;
     Mem mem{h->custom_al ? &h->al : nullptr, h->stream};
     mem.put(h->pool, h->pool_bytes);
-    mem.put(h->row_mode, (size_t)std::max<int64_t>(h->n_rows, 1));
     delete h;
     return LF_OK;
 }

@@ -38,6 +38,12 @@ struct BucketDev {
     int32_t task_slots; // slots per task: 32 (W <= 32), W (W <= 2^kPieceLog2) or 2^kPieceLog2
     int32_t piece_log2; // W >= 32: a CELL row is 2^piece_log2 tasks of <= 2^kPieceLog2 slots
     int32_t pad_;
+    int64_t n_real_rows; // CELL rows before block padding
+    int64_t n_rows_pad;  // CELL rows after block padding
+};
+// max width exponents e_p passed by value to the build kernels
+struct WidthArg {
+    int8_t e[LF_MAX_PARTS];
 };
 
 // Stats the configure kernels accumulate (device, zero-initialised).
@@ -53,7 +59,6 @@ inline size_t stats_bytes(int P) { return offsetof(StatsDev, part) + (size_t)P *
 // ---- launchers (kernels in csrc/kernels/*.cu) ----
 uint32_t mask_slots(int64_t n_cols);  // words of the column-mask array (power of two >= K)
 size_t stats_scratch_bytes(int64_t n_rows, int64_t nnz, int P);  // t0 per segment + tile -> row map
-cudaError_t launch_features(const lf_csr &A, StatsDev *d_stats, cudaStream_t s);  // len_* only
 cudaError_t launch_stats(const lf_csr &A, int P, StatsDev *d_stats, uint32_t *d_colmask, uint8_t *d_t0seg,
                          cudaStream_t s);
 
@@ -97,10 +102,14 @@ enum : uint8_t {
 };
 
 cudaError_t launch_seg(const lf_csr &A, int P, int32_t *seg_rel, cudaStream_t s);
-cudaError_t launch_bucket_count(const lf_csr &A, int P, const int8_t *e, const BuildScratch &sc,
+cudaError_t launch_bucket_count(const lf_csr &A, int P, const WidthArg &e, const BuildScratch &sc,
                                 int32_t *row_cnt, cudaStream_t s);
+// padding rows (n_real_rows .. n_rows_pad of every bucket): rowInd / tag -1,
+// src_cnt 0; and the n_ctr queue counters zeroed
+cudaError_t launch_pad_init(const BucketDev *bk, int nb, int32_t *row_ind, int32_t *row_tag, int32_t *src_cnt,
+                            unsigned long long *ctr, int n_ctr, cudaStream_t s);
 cudaError_t launch_tile_scan(int P, const BuildScratch &sc, cudaStream_t s);
-cudaError_t launch_bucket_place(const lf_csr &A, int P, const int8_t *e, const BuildScratch &sc,
+cudaError_t launch_bucket_place(const lf_csr &A, int P, const WidthArg &e, const BuildScratch &sc,
                                 const int32_t *row_cnt, int32_t *row_ind, int32_t *row_tag, uint8_t *row_mode,
                                 cudaStream_t s);
 cudaError_t launch_run_bounds(const BucketDev *bk_w, int nb_w, int64_t n_tasks_w, const int32_t *row_tag,
