@@ -190,8 +190,12 @@ typedef struct lf_cell lf_cell; /* opaque handle */
  * (section 5.3) to pick e_p; k_p = e_p + block_mult_log2.
  *   A      (host struct of device pointers)   J >= 1   opts may be NULL
  *   out    (host) receives the parameters     stats (host) may be NULL
- * Synchronises stream s twice when the predictor runs (features, then
- * statistics: two small device-to-host copies), once otherwise.
+ * The statistics pass also yields the features, so with the predictor on
+ * and nnz <= 2^25 it runs once for P = 1 before the prediction and again
+ * only if another P is predicted; larger matrices read the features from
+ * row_ptr first.  When the fixed CSR format is chosen (use_cell = 0) no
+ * CELL statistics are computed (stats: features only, tables zero).
+ * Synchronises stream s once or twice (small device-to-host copies).
  * Errors: LF_ERR_INVALID_ARG for bad sizes / pointers / options. */
 LF_API lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts *opts, lf_cell_params *out,
                             lf_configure_stats *stats, lf_stream_t s);

@@ -282,6 +282,18 @@ __host__ __device__ constexpr uint32_t inv_odd(uint32_t a) {
 }
 static_assert(kHashOdd * inv_odd(kHashOdd) == 1u, "hash inverse");
 
+// 32 x 32 bit-matrix transpose across a warp: on return, bit j of lane t's
+// word is bit t of lane j's input word (five shuffle-and-swap rounds).
+__device__ __forceinline__ uint32_t transpose32(uint32_t x, int lane) {
+    const uint32_t lo[5] = {0x0000FFFFu, 0x00FF00FFu, 0x0F0F0F0Fu, 0x33333333u, 0x55555555u};
+#pragma unroll
+    for (int i = 0, k = 16; i < 5; i++, k >>= 1) {
+        const uint32_t y = __shfl_xor_sync(kFull, x, k);
+        x = (lane & k) ? (x & ~lo[i]) | ((y & ~lo[i]) >> k) : (x & lo[i]) | ((y & lo[i]) << k);
+    }
+    return x;
+}
+
 __global__ void __launch_bounds__(kThreads) stats_cols_kernel(const uint32_t *__restrict__ mask, int64_t n_cols,
                                                               int64_t S, int P, StatsDev *st, uint32_t kmask) {
     extern __shared__ unsigned long long sh[];  // Un_s[P][32], Hb_s[P][32]
@@ -320,16 +332,10 @@ __global__ void __launch_bounds__(kThreads) stats_cols_kernel(const uint32_t *__
                 flush();
                 cur_p = pp;
             }
-            const uint32_t mm = mine ? m : 0u;
-#pragma unroll
-            for (int t = 0; t < 32; t++) {
-                const unsigned un = __popc(__ballot_sync(kFull, (mm >> t) & 1u));
-                const unsigned nh = __popc(__ballot_sync(kFull, mine && hb == t));
-                if (lane == t) {
-                    my_un += un;
-                    my_hb += nh;
-                }
-            }
+            // bit-matrix transpose: lane t then holds bit t of every lane's
+            // word, so one popc per lane counts the group's columns
+            my_un += __popc(transpose32(mine ? m : 0u, lane));
+            my_hb += __popc(transpose32(mine ? 1u << hb : 0u, lane));
         }
     }
     flush();
@@ -364,6 +370,37 @@ uint32_t mask_slots(int64_t n_cols) {
     uint64_t m = 1;
     while ((int64_t)m < n_cols) m <<= 1;
     return (uint32_t)m;
+}
+
+namespace {
+
+// Table 2 row-length statistics alone: the features the
+// predictor needs BEFORE P is known (section 5.1-5.2), from row_ptr only
+// (8 B per row).  One thread per row, warp then block reduction, one set of
+// 64-bit atomics per block.  (Used when the statistics pass is too long to
+// run speculatively for P = 1, see lf_cell_configure.)
+__global__ void __launch_bounds__(kThreads) features_kernel(const int64_t *__restrict__ row_ptr, int64_t n_rows,
+                                                            StatsDev *st) {
+    unsigned long long mn = ~0ull, mx = 0, sum = 0, sq = 0;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_rows; i += stride) {
+        const unsigned long long len = (unsigned long long)(__ldg(row_ptr + i + 1) - __ldg(row_ptr + i));
+        mn = min(mn, len);
+        mx = max(mx, len);
+        sum += len;
+        sq += len * len;
+    }
+    block_len_stats(mn, mx, sum, sq, st);
+}
+
+}  // namespace
+
+cudaError_t launch_features(const lf_csr &A, StatsDev *d_stats, cudaStream_t s) {
+    if (A.n_rows <= 0) return cudaSuccess;
+    const int64_t want = (A.n_rows + kThreads - 1) / kThreads;
+    const int grid = (int)std::min<int64_t>(want, (int64_t)num_sms() * 8);
+    features_kernel<<<grid, kThreads, 0, s>>>(A.row_ptr, A.n_rows, d_stats);
+    return cudaGetLastError();
 }
 
 cudaError_t launch_stats(const lf_csr &A, int P, StatsDev *d_stats, uint32_t *d_colmask, uint8_t *d_t0seg,

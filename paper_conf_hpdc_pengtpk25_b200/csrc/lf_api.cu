@@ -192,13 +192,32 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
         return LF_OK;
     };
     // predictor (sections 5.1-5.2): it needs the Table 2 row-length features
-    // before P is known.  The statistics pass computes them too, so it runs
-    // once speculatively for P = 1 (the forced P if given) and only again if
-    // the predictor picks another P -- one pass and one sync in the common case.
+    // before P is known.  The statistics pass computes them too, so for
+    // matrices up to kSpeculateNnz nonzeros it runs once speculatively for
+    // P = 1 (the forced P if given) and again only if the predictor picks
+    // another P: one pass and one sync in the common case.  Larger matrices
+    // (where a wasted pass costs more than a sync) read the features from
+    // row_ptr alone first.
+    constexpr int64_t kSpeculateNnz = int64_t(1) << 25;
     int P = o.force_parts ? o.force_parts : 1;
     int use_cell = o.force_format == 2 ? 0 : 1;
-    if (lf_status st = run_stats(P)) return st;
-    if (o.force_parts == 0 || o.force_format == 0) {
+    const bool predict = o.force_parts == 0 || o.force_format == 0;
+    bool have = false;
+    if (predict) {
+        if (o.force_parts != 0 || A->nnz <= kSpeculateNnz) {
+            if (lf_status st = run_stats(P)) return st;
+            have = true;
+        } else {
+            lf::StatsDev *d_f = nullptr;
+            const size_t fb = lf::stats_bytes(0);
+            LF_CUDA(cudaMallocAsync(&d_f, fb, s));
+            LF_CUDA(cudaMemsetAsync(d_f, 0, fb, s));
+            LF_CUDA(cudaMemsetAsync(&d_f->len_min, 0xFF, sizeof(unsigned long long), s));
+            LF_CUDA(lf::launch_features(*A, d_f, s));
+            LF_CUDA(cudaMemcpyAsync(h_st, d_f, fb, cudaMemcpyDeviceToHost, s));
+            LF_CUDA(cudaFreeAsync(d_f, s));
+            LF_CUDA(cudaStreamSynchronize(s));
+        }
         double f[8];
         table2_features(*A, J, *h_st, f);
         int32_t pu = 1, pp = 1;
@@ -206,9 +225,26 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
         if (o.force_format == 0) use_cell = pu;
         if (o.force_parts == 0 && pp != P) {
             P = pp;
-            if (lf_status st = run_stats(P)) return st;
+            have = false;
         }
     }
+    // the fixed CSR format needs no CELL composition (section 5: the
+    // predictor picks the format first): no statistics pass then
+    const bool need_stats = use_cell != 0;
+    if (!have && need_stats)
+        if (lf_status st = run_stats(P)) return st;
+    if (!have && !need_stats && !predict) {  // forced CSR: the features alone
+        lf::StatsDev *d_f = nullptr;
+        const size_t fb = lf::stats_bytes(0);
+        LF_CUDA(cudaMallocAsync(&d_f, fb, s));
+        LF_CUDA(cudaMemsetAsync(d_f, 0, fb, s));
+        LF_CUDA(cudaMemsetAsync(&d_f->len_min, 0xFF, sizeof(unsigned long long), s));
+        LF_CUDA(lf::launch_features(*A, d_f, s));
+        LF_CUDA(cudaMemcpyAsync(h_st, d_f, fb, cudaMemcpyDeviceToHost, s));
+        LF_CUDA(cudaFreeAsync(d_f, s));
+        LF_CUDA(cudaStreamSynchronize(s));
+    }
+    if (!have && !need_stats) std::memset(h_st->part, 0, sizeof(h_st->part[0]) * (size_t)P);
     const lf::StatsDev &st = *h_st;
 
     lf_configure_stats local;

@@ -59,6 +59,7 @@ inline size_t stats_bytes(int P) { return offsetof(StatsDev, part) + (size_t)P *
 // ---- launchers (kernels in csrc/kernels/*.cu) ----
 uint32_t mask_slots(int64_t n_cols);  // words of the column-mask array (power of two >= K)
 size_t stats_scratch_bytes(int64_t n_rows, int64_t nnz, int P);  // t0 per segment + tile -> row map
+cudaError_t launch_features(const lf_csr &A, StatsDev *d_stats, cudaStream_t s);  // len_* only
 cudaError_t launch_stats(const lf_csr &A, int P, StatsDev *d_stats, uint32_t *d_colmask, uint8_t *d_t0seg,
                          cudaStream_t s);
 
