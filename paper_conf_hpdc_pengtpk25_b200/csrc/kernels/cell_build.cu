@@ -212,10 +212,13 @@ __global__ void pad_init_kernel(const BucketDev *__restrict__ bk, int nb, int32_
 
 constexpr int kSlotThreads = 256;
 constexpr int kMaxSmemBuckets = 2048;
-constexpr int kSlotsPerLane = 4;                    // consecutive slots: one 16-byte store each
+#ifndef LF_SLOTS_PER_LANE
+#define LF_SLOTS_PER_LANE 4  // measured: 8 same, 16 slower (c2)
+#endif
+constexpr int kSlotsPerLane = LF_SLOTS_PER_LANE;    // consecutive slots per lane: 16-byte stores
 constexpr int kSlotsPerWarp = 32 * kSlotsPerLane;   // a warp's chunk
 
-// A warp fills 128 consecutive slots per chunk, 4 per lane (vector stores).
+// A warp fills 32 * kSlotsPerLane consecutive slots per chunk (16-byte stores).
 // The bucket of the chunk is found once (warp-uniform binary search over the
 // bucket slot offsets in shared memory); a chunk that straddles buckets
 // falls back to a per-slot search.  Slot s of bucket b is position
@@ -280,8 +283,11 @@ __global__ void __launch_bounds__(kSlotThreads)
             v[k] = real ? __ldg(val + pos[k] + w[k]) : 0.0f;
         }
         if (s0 + kSlotsPerLane <= n_slots) {
-            __stcs(reinterpret_cast<int4 *>(col_out + s0), make_int4(c[0], c[1], c[2], c[3]));
-            __stcs(reinterpret_cast<float4 *>(val_out + s0), make_float4(v[0], v[1], v[2], v[3]));
+#pragma unroll
+            for (int k = 0; k < kSlotsPerLane; k += 4) {
+                __stcs(reinterpret_cast<int4 *>(col_out + s0 + k), make_int4(c[k], c[k + 1], c[k + 2], c[k + 3]));
+                __stcs(reinterpret_cast<float4 *>(val_out + s0 + k), make_float4(v[k], v[k + 1], v[k + 2], v[k + 3]));
+            }
         } else {
 #pragma unroll
             for (int k = 0; k < kSlotsPerLane; k++)
@@ -387,7 +393,7 @@ cudaError_t launch_slot_fill(const lf_csr &A, const BucketDev *d_buckets, int nb
                              const BuildScratch &sc, int32_t *col_out, float *val_out, cudaStream_t s) {
     if (n_slots == 0) return cudaSuccess;
     if (nb > kMaxSmemBuckets) return cudaErrorInvalidValue;
-    static_assert(kSlotsPerLane == 4, "vector stores");
+    static_assert(kSlotsPerLane % 4 == 0, "vector stores");
     slot_fill_kernel<<<grid_for((n_slots + kSlotsPerLane - 1) / kSlotsPerLane, kSlotThreads), kSlotThreads, 0, s>>>(
         A.col_ind, A.val, d_buckets, nb, n_slots, sc.src_pos, sc.src_cnt, col_out, val_out);
     return cudaGetLastError();
