@@ -146,6 +146,9 @@ typedef struct lf_configure_stats {
     int64_t Unat[LF_MAX_PARTS][32];
     int64_t Utop[LF_MAX_PARTS][32];
     int64_t cost[LF_MAX_PARTS][32];
+    double group_union_ratio; /* sampled: distinct columns / nonzeros of groups of 4 consecutive rows */
+    int32_t spmm_grouped;     /* 1: lf_cell_build given these stats makes lf_spmm take the grouped path */
+    int32_t pad_;
 } lf_configure_stats;
 
 /* One CELL bucket (Fig. 4).  Buckets are stored

@@ -853,6 +853,181 @@ cudaError_t run_csr_j(const lf_csr &A, const float *B, int64_t ldb, int J, float
                                        : run_csr<VEC, G, NV, false>(A, B, ldb, J, C, ldc, s);
 }
 
+// ---- grouped (column-merged) path -----------------------------------------
+// Eq. 7 charges a bucket U.J for its B reads (U = distinct columns):
+// the cost model assumes every distinct B row is fetched once.  The per-slot
+// path above fetches one B row per nonzero instead, so on matrices whose
+// consecutive rows share columns (banded / FEM / stencil) it gathers each
+// B row several times (27-point stencil: every column is in 3 consecutive
+// rows).  The grouped path takes kGR consecutive CELL rows of a bucket (W <=
+// 32) per warp, merges their columns in a per-warp shared-memory hash table
+// (key = column, value = the kGR row values), gathers each DISTINCT B row
+// once and applies it to all kGR row accumulators held in registers.
+// Measured B-row gathers drop to the group's union (stencil: 0.50 of nnz at
+// kGR = 4).  Rows are written like the per-slot path: plain store when the
+// CELL row is the whole C row, red.add otherwise (kRowRun rows pre-zeroed).
+constexpr int kGR = kGroupRows;  // CELL rows per group
+constexpr int kHT = 256;   // hash slots per warp (>= kGR * 32 distinct columns)
+struct GroupStage {
+    int32_t key[kHT];      // column in hash slot, -1 = free
+    int32_t idx_of[kHT];   // entry index of the slot's column
+    int32_t hslot[kGR * 32];
+    int32_t ckey[kGR * 32];   // entry k: column ...
+    float4 cval[kGR * 32];    // ... and its value in each of the kGR rows (0 if absent)
+};
+#ifndef LF_GROUP_MIN_BLOCKS
+#define LF_GROUP_MIN_BLOCKS 4
+#endif
+
+__device__ __forceinline__ float *f4c(float4 &v, int r) { return reinterpret_cast<float *>(&v) + r; }
+
+template <int G, int NV, bool FULL>
+__global__ void __launch_bounds__(kWarpsPerBlock * 32, LF_GROUP_MIN_BLOCKS) cell_spmm_grouped_kernel(const SpmmArgs a) {
+    using Cx = Ctx<4, G, NV, FULL>;
+    using V = typename Cx::V;
+    using VT = typename Cx::VT;
+    using L = Layout<4, G, NV>;
+    constexpr int U = 4;  // distinct columns in flight per lane group
+    __shared__ __align__(16) GroupStage gs_all[kWarpsPerBlock];
+    const int lane = threadIdx.x & 31;
+    const int w = threadIdx.x >> 5;
+    GroupStage &gs = gs_all[w];
+    for (int q = lane; q < kHT; q += 32) gs.key[q] = -1;
+    __syncwarp();
+    const uint64_t pol = policy_evict_first();
+    const Cx cx{a.B, a.ldb, a.C, a.ldc, a.J, 0, lane / L::LPR, lane % L::LPR, pol};
+    const int64_t nw = (int64_t)gridDim.x * kWarpsPerBlock;
+    zero_rows_warp(a.row_mode, a.n_rows, a.C, a.ldc, a.J, true, 1u << kRowEmpty,
+                   (int64_t)blockIdx.x * kWarpsPerBlock + w, nw, lane, pol);
+    const unsigned lt = (1u << lane) - 1u;
+    const int64_t n = a.n_groups;
+    int bcur = 0;
+    int sz = claim_size(n, 0, nw);
+    int64_t g = claim_get(claim_issue(a.ctr + 1, sz, lane));
+    int64_t gend = min(g + sz, n);
+    while (g < n) {
+        while (bcur + 1 < a.nb_g && __ldg(&a.bk_g[bcur + 1].task_off) <= g) bcur++;
+        const BucketDev *bk = a.bk_g + bcur;
+        const int t = __ldg(&bk->t);
+        const int W = 1 << t;
+        const int64_t r0 = (g - __ldg(&bk->task_off)) * kGR;  // first CELL row of the group in the bucket
+        const int nr = (int)min((int64_t)kGR, __ldg(&bk->n_rows_pad) - r0);
+        const int64_t row0 = __ldg(&bk->row_off) + r0;
+        const int64_t slot0 = __ldg(&bk->slot_off) + r0 * W;
+        const int32_t tag_l = lane < nr ? __ldg(a.row_tag + row0 + lane) : -1;
+        // the group's slots: lane j holds slot j of each row (W <= 32)
+        int32_t c[kGR];
+        float v[kGR];
+#pragma unroll
+        for (int r = 0; r < kGR; r++) {
+            const bool in = r < nr && lane < W;
+            c[r] = in ? ld_stream(a.col + slot0 + (int64_t)r * W + lane, pol) : -1;
+            v[r] = in ? ld_stream(a.val + slot0 + (int64_t)r * W + lane, pol) : 0.f;
+        }
+        // merge: every real slot's column is inserted (linear probing); a new
+        // column gets the next entry index in (row, lane) order, so entries
+        // -- and the gather / summation order -- are deterministic; then each
+        // slot adds its value into component r of its column's entry
+        int n_u = 0;
+#pragma unroll
+        for (int r = 0; r < kGR; r++) {
+            bool need = c[r] >= 0, ins = false;
+            int h = (int)(((uint32_t)c[r] * 0x9E3779B1u) >> 24);
+            while (__any_sync(kFull, need)) {
+                if (need) {
+                    const int prev = atomicCAS(&gs.key[h], -1, c[r]);
+                    if (prev == -1) ins = true;
+                    if (prev == -1 || prev == c[r]) need = false;
+                    else h = (h + 1) & (kHT - 1);
+                }
+            }
+            const unsigned im = __ballot_sync(kFull, ins);
+            if (ins) {
+                const int k = n_u + __popc(im & lt);
+                gs.idx_of[h] = k;
+                gs.hslot[k] = h;
+                gs.ckey[k] = c[r];
+                gs.cval[k] = make_float4(0.f, 0.f, 0.f, 0.f);
+            }
+            n_u += __popc(im);
+            __syncwarp();
+            if (c[r] >= 0) atomicAdd(f4c(gs.cval[gs.idx_of[h]], r), v[r]);
+        }
+        __syncwarp();
+        // gather each distinct B row once; lane group gi takes entries gi, gi + G, ...
+        VT acc[kGR][NV];
+#pragma unroll
+        for (int r = 0; r < kGR; r++) cx.zero(acc[r]);
+        for (int k0 = 0; k0 < n_u; k0 += G * U) {
+            VT b[U][NV];
+            float4 vv[U];
+#pragma unroll
+            for (int u = 0; u < U; u++) {
+                const int k = k0 + u * G + cx.g;
+                const bool ok = k < n_u;
+                vv[u] = ok ? gs.cval[k] : make_float4(0.f, 0.f, 0.f, 0.f);
+                cx.gather(cx.rowaddr(ok ? gs.ckey[k] : -1), b[u]);
+            }
+#pragma unroll
+            for (int u = 0; u < U; u++)
+#pragma unroll
+                for (int m = 0; m < NV; m++) {
+                    V::fma(acc[0][m], vv[u].x, b[u][m]);
+                    V::fma(acc[1][m], vv[u].y, b[u][m]);
+                    V::fma(acc[2][m], vv[u].z, b[u][m]);
+                    V::fma(acc[3][m], vv[u].w, b[u][m]);
+                }
+        }
+        for (int k = lane; k < n_u; k += 32) gs.key[gs.hslot[k]] = -1;  // free the used slots
+#pragma unroll
+        for (int r = 0; r < kGR; r++) {
+            cx.reduce_groups(acc[r]);
+            const int32_t tag = __shfl_sync(kFull, tag_l, r);
+            if (r < nr && tag >= 0 && cx.g == 0) cx.write(tag_row(tag), tag_whole(tag), acc[r]);
+        }
+        __syncwarp();
+        if (++g >= gend) {
+            sz = claim_size(n, g, nw);
+            g = claim_get(claim_issue(a.ctr + 1, sz, lane));
+            gend = min(g + sz, n);
+        }
+    }
+    if (lane == 0) {  // the last warp out resets the queue counters (as cell_spmm_kernel)
+        __threadfence();
+        if (atomicAdd(a.ctr + 2, 1ull) == (unsigned long long)gridDim.x * kWarpsPerBlock - 1) {
+            __threadfence();
+            a.ctr[0] = 0;
+            a.ctr[1] = 0;
+            a.ctr[2] = 0;
+        }
+    }
+}
+
+template <int G, int NV, bool FULL>
+cudaError_t run_grouped(const SpmmArgs &a, cudaStream_t s) {
+    static int cap = 0;
+    auto fn = cell_spmm_grouped_kernel<G, NV, FULL>;
+    if (!cap) cap = resident_blocks(fn);
+    const int64_t want = std::max<int64_t>((a.n_groups + kWarpsPerBlock - 1) / kWarpsPerBlock,
+                                           (a.n_rows + 32 * kWarpsPerBlock - 1) / (32 * kWarpsPerBlock));
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(cap, want));
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)grid);
+    cfg.blockDim = dim3(kWarpsPerBlock * 32);
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, fn, a);
+}
+
+template <int G, int NV>
+cudaError_t run_grouped_j(const SpmmArgs &a, cudaStream_t s) {
+    return a.J == Layout<4, G, NV>::JT ? run_grouped<G, NV, true>(a, s) : run_grouped<G, NV, false>(a, s);
+}
+
 bool vec4_ok(const float *B, int64_t ldb, const float *C, int64_t ldc, int J) {
     return J % 4 == 0 && ldb % 4 == 0 && ldc % 4 == 0 && ((uintptr_t)B & 15) == 0 && ((uintptr_t)C & 15) == 0;
 }
@@ -871,9 +1046,20 @@ cudaError_t zero_red_rows(const SpmmArgs &a, bool tiled, cudaStream_t s) {
     return cudaGetLastError();
 }
 
+bool grouped_ok(const SpmmArgs &a) {
+    return a.grouped && a.nb_g > 0 && vec4_ok(a.B, a.ldb, a.C, a.ldc, a.J) && a.J <= 128;
+}
+
 cudaError_t launch_cell_spmm(const SpmmArgs &a, cudaStream_t s) {
     if (a.J == 0 || a.n_rows == 0) return cudaSuccess;
     const bool v4 = vec4_ok(a.B, a.ldb, a.C, a.ldc, a.J);
+    if (grouped_ok(a)) {  // runs of folded rows are split across groups: red.add, pre-zeroed
+        cudaError_t e = zero_red_rows(a, true, s);
+        if (e != cudaSuccess) return e;
+        if (a.J <= 32) return run_grouped_j<4, 1>(a, s);
+        if (a.J <= 64) return run_grouped_j<2, 1>(a, s);
+        return run_grouped_j<1, 1>(a, s);
+    }
     const bool tiled = v4 ? a.J > 512 : a.J > 128;
     cudaError_t e = zero_red_rows(a, tiled, s);
     if (e != cudaSuccess) return e;

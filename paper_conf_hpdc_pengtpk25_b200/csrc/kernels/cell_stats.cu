@@ -403,6 +403,58 @@ cudaError_t launch_features(const lf_csr &A, StatsDev *d_stats, cudaStream_t s) 
     return cudaGetLastError();
 }
 
+// Grouped-path heuristic (cell_spmm.cu "grouped path"): on kGroupSamples
+// groups of kGroupRows consecutive rows spread evenly over A (rows of at most
+// 32 nonzeros; a group with a longer row is skipped), the number of DISTINCT
+// columns of the group and its nonzeros, summed.  Their ratio says how many
+// B-row gathers merging the group's columns saves.  A warp per group, the
+// distinct columns counted in a per-warp shared-memory hash set.
+constexpr int kGroupSamples = 2048;
+__global__ void __launch_bounds__(256) group_sample_kernel(const int64_t *__restrict__ row_ptr,
+                                                           const int32_t *__restrict__ col, int64_t n_rows,
+                                                           StatsDev *st) {
+    __shared__ int32_t hs[8][256];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    for (int q = lane; q < 256; q += 32) hs[w][q] = -1;
+    __syncwarp();
+    const int64_t smp = (int64_t)blockIdx.x * 8 + w;
+    const int64_t n_groups = n_rows / kGroupRows;
+    if (smp >= kGroupSamples || n_groups == 0) return;
+    const int64_t i0 = (smp * n_groups / kGroupSamples) * kGroupRows;
+    const int64_t base = row_ptr[0];
+    int64_t b[kGroupRows], l[kGroupRows];
+    bool ok = true;
+#pragma unroll
+    for (int r = 0; r < kGroupRows; r++) {
+        b[r] = row_ptr[i0 + r] - base;
+        l[r] = row_ptr[i0 + r + 1] - base - b[r];
+        ok = ok && l[r] <= 32;
+    }
+    if (!ok) return;
+    const int32_t *colb = col + base;
+    unsigned n_u = 0, n_nz = 0;
+#pragma unroll
+    for (int r = 0; r < kGroupRows; r++) {
+        const int32_t c = lane < l[r] ? colb[b[r] + lane] : -1;
+        bool need = c >= 0, ins = false;
+        int h = (int)(((uint32_t)c * 0x9E3779B1u) >> 24);
+        while (__any_sync(kFull, need)) {
+            if (need) {
+                const int prev = atomicCAS(&hs[w][h], -1, c);
+                if (prev == -1) ins = true;
+                if (prev == -1 || prev == c) need = false;
+                else h = (h + 1) & 255;
+            }
+        }
+        n_u += __popc(__ballot_sync(kFull, ins));
+        n_nz += (unsigned)l[r];
+    }
+    if (lane == 0) {
+        atomicAdd(&st->grp_union, (unsigned long long)n_u);
+        atomicAdd(&st->grp_nnz, (unsigned long long)n_nz);
+    }
+}
+
 cudaError_t launch_stats(const lf_csr &A, int P, StatsDev *d_stats, uint32_t *d_colmask, uint8_t *d_t0seg,
                          cudaStream_t s) {
     const int64_t S = A.n_cols > 0 ? (A.n_cols + P - 1) / P : 1;
@@ -421,6 +473,8 @@ cudaError_t launch_stats(const lf_csr &A, int P, StatsDev *d_stats, uint32_t *d_
                                                                     tile_row, tile_pos, tiles, d_colmask,
                                                                     mask_slots(A.n_cols) - 1);
     }
+    if (A.n_rows >= kGroupRows && A.nnz > 0)
+        group_sample_kernel<<<kGroupSamples / 8, 256, 0, s>>>(A.row_ptr, A.col_ind, A.n_rows, d_stats);
     if (A.n_cols > 0) {
         const int64_t want = ((int64_t)mask_slots(A.n_cols) + kThreads - 1) / kThreads;
         const int grid = (int)std::min<int64_t>(want, (int64_t)num_sms() * 8);

@@ -117,6 +117,9 @@ void table2_features(const lf_csr &A, int32_t J, const lf::StatsDev &st, double 
     f[7] = (double)J;
 }
 
+constexpr double kGroupedMaxRatio = 0.35;   // grouped path: distinct / nonzeros of 4-row groups
+constexpr double kGroupedMinMeanLen = 16.0; // ... and mean row length
+
 // Algorithm 3 in exponent space (reading R8) over eq. 7 costs.
 int alg3(const int64_t *cost, int hi) {
     int lo = 0;
@@ -284,6 +287,18 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
         prm.max_width_log2[p] = (int8_t)e;
         prm.block_nnz_log2[p] = (int8_t)std::min(e + o.block_mult_log2, LF_MAX_LOG2);
     }
+    // grouped SpMM path (cell_spmm.cu): worth it when consecutive rows share
+    // most of their columns and the rows are long enough for a group to
+    // amortise the column merge (measured on B200: banded / dense-block rows
+    // of 25-32 nonzeros at ratio <= 0.28 gain 1.3-1.45x, the 27-point stencil
+    // at 0.50 and rows of 8 lose); needs every W_p <= 32 and J <= 128
+    cs.group_union_ratio = st.grp_nnz ? (double)st.grp_union / (double)st.grp_nnz : 1.0;
+    bool narrow = true;
+    for (int p = 0; p < P; p++) narrow = narrow && prm.max_width_log2[p] <= 5;
+    cs.spmm_grouped = (use_cell && narrow && J <= 128 && cs.group_union_ratio <= kGroupedMaxRatio &&
+                       cs.features[3] >= kGroupedMinMeanLen)
+                          ? 1
+                          : 0;
     *out = prm;
     return LF_OK;
 }
@@ -310,6 +325,7 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
 
     lf_cell *h = new lf_cell();
     h->params = *params;
+    h->grouped = stats ? stats->spmm_grouped : 0;
     h->n_rows = A->n_rows;
     h->n_cols = A->n_cols;
     h->nnz = A->nnz;
@@ -393,8 +409,22 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
         h->n_slots = S_tot;
         h->nb_n = (int)bn.size();
         h->nb_w = (int)bw.size();
+        const int nb_all = (int)h->h_buckets.size();
         h->h_buckets.insert(h->h_buckets.end(), bn.begin(), bn.end());
         h->h_buckets.insert(h->h_buckets.end(), bw.begin(), bw.end());
+        // grouped SpMM path (every W <= 32): the buckets again, task_off
+        // counting groups of kGroupRows CELL rows
+        bool narrow = nb_all > 0;
+        for (int q = 0; q < nb_all; q++) narrow = narrow && h->h_buckets[q].t <= 5;
+        if (narrow) {
+            for (int q = 0; q < nb_all; q++) {
+                lf::BucketDev d = h->h_buckets[q];
+                d.task_off = h->n_groups;
+                h->n_groups += (d.n_rows_pad + lf::kGroupRows - 1) / lf::kGroupRows;
+                h->h_buckets.push_back(d);
+            }
+            h->nb_g = nb_all;
+        }
         if (h->buckets.size() > 2048) return fail(LF_ERR_UNSUPPORTED, "more than 2048 buckets");
         return LF_OK;
     };
@@ -518,7 +548,9 @@ lf_status lf_spmm(const lf_cell *h, const float *B, int64_t ldb, int32_t J, floa
                    h->slots_n, h->slots_w, 0, h->row_mode, h->n_rows, h->run_bound,
                    h->ctr_ring + 4 * (h->launch_seq.fetch_add(1, std::memory_order_relaxed) % kCtrSlots), h->col_ind, h->val,
                    h->row_tag,
-                   B, ldb, C, ldc, J};
+                   B, ldb, C, ldc, J,
+                   h->d_buckets + nb + h->nb_n + h->nb_w, h->nb_g, h->grouped, h->n_groups};
+    if (const char *g = std::getenv("LF_GROUPED")) a.grouped = g[0] == '1';
     LF_CUDA(lf::launch_cell_spmm(a, s));
     return LF_OK;
 }

@@ -52,6 +52,7 @@ struct StatsPart {
 };
 struct StatsDev {
     unsigned long long len_min, len_max, len_sum, len_sumsq;  // row lengths
+    unsigned long long grp_union, grp_nnz;  // sampled groups of kGroupRows rows: distinct columns, nonzeros
     StatsPart part[LF_MAX_PARTS];  // only the first P are cleared / copied back
 };
 inline size_t stats_bytes(int P) { return offsetof(StatsDev, part) + (size_t)P * sizeof(StatsPart); }
@@ -94,6 +95,8 @@ constexpr int kWideChunk = LF_WIDE_CHUNK;
 #define LF_PIECE_LOG2 10
 #endif
 constexpr int kPieceLog2 = LF_PIECE_LOG2;
+// CELL rows per group of the grouped SpMM path (cell_spmm.cu)
+constexpr int kGroupRows = 4;
 // row_mode[i]: how C row i is produced
 enum : uint8_t {
     kRowPlain = 0,  // one CELL row, plain store
@@ -138,6 +141,11 @@ struct SpmmArgs {
     float *C;
     int64_t ldc;
     int J;
+    // grouped path (cell_spmm.cu): every bucket W <= 32, task_off = first group
+    const BucketDev *bk_g;
+    int nb_g;
+    int grouped;  // use it (when J and the alignment allow)
+    int64_t n_groups;
 };
 cudaError_t launch_cell_spmm(const SpmmArgs &a, cudaStream_t s);  // pre-zeroes kRowRed rows itself
 cudaError_t launch_csr_spmm(const lf_csr &A, const float *B, int64_t ldb, int J, float *C, int64_t ldc,
@@ -159,7 +167,10 @@ struct lf_cell {
     int32_t *row_tag = nullptr;  // (row << 3) | S,F,L flags (cell_spmm.cu); -1 = padding
     uint8_t *row_mode = nullptr;  // [n_rows] kRow* (how each C row is produced)
     uint8_t *run_bound = nullptr; // [n_tasks_w + 1] (in the pool)
-    lf::BucketDev *d_buckets = nullptr;  // [nb] all, then [nb_n] W < 32 class, then [nb_w] W >= 32 class
+    lf::BucketDev *d_buckets = nullptr;  // [nb] all, [nb_n] W < 32 class, [nb_w] W >= 32 class, [nb_g] grouped
+    int nb_g = 0;            // grouped-path buckets (= nb when every W <= 32, else 0)
+    int64_t n_groups = 0;
+    int grouped = 0;         // lf_spmm takes the grouped path
     // work-queue counters, kCtrSlots slots of 4 (wide, narrow, warps done, -)
     // in the pool: launch k uses slot k % kCtrSlots and its last warp resets
     // it, so lf_spmm needs no allocation or memset per call

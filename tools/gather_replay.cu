@@ -14,17 +14,31 @@
 
 #define CK(x) do { cudaError_t e = (x); if (e != cudaSuccess) { printf("%s: %s\n", #x, cudaGetErrorString(e)); exit(1); } } while (0)
 
-template <int U, int MODE>
+// ILV = 0: each warp replays a contiguous range of 32-index chunks (like the
+// SpMM's per-warp claims); ILV = 1: each BLOCK takes a contiguous range and
+// its 8 warps interleave over it (chunk start + w, start + w + 8, ...), so
+// consecutive chunks -- consecutive rows -- are gathered on one SM at once
+template <int U, int MODE, int ILV = 0>
 __global__ void __launch_bounds__(256) replay(const float4 *__restrict__ tab, const int *__restrict__ idx, int64_t n_idx,
                                               int row_f4, float4 *__restrict__ out) {
   const int lane = threadIdx.x & 31;
   const int64_t w = (blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5;
   const int64_t nw = (gridDim.x * (int64_t)blockDim.x) >> 5;
   float4 acc = make_float4(0, 0, 0, 0);
-  // contiguous range of 32-index chunks per warp (like the SpMM's claims)
   const int64_t n_ch = (n_idx + 31) / 32;
-  const int64_t per = (n_ch + nw - 1) / nw;
-  for (int64_t ch = w * per; ch < min(n_ch, (w + 1) * per); ch++) {
+  int64_t c_beg, c_end, c_step;
+  if (ILV) {
+    const int64_t wpb = blockDim.x >> 5, per = (n_ch + gridDim.x - 1) / gridDim.x;
+    c_beg = blockIdx.x * per + (threadIdx.x >> 5);
+    c_end = min(n_ch, (int64_t)(blockIdx.x + 1) * per);
+    c_step = wpb;
+  } else {
+    const int64_t per = (n_ch + nw - 1) / nw;
+    c_beg = w * per;
+    c_end = min(n_ch, (w + 1) * per);
+    c_step = 1;
+  }
+  for (int64_t ch = c_beg; ch < c_end; ch += c_step) {
     const int64_t q = ch * 32;
     int my = q + lane < n_idx ? __ldcs(idx + q + lane) : 0;
 #pragma unroll
@@ -48,13 +62,13 @@ __global__ void __launch_bounds__(256) replay(const float4 *__restrict__ tab, co
   if (acc.x + acc.y + acc.z + acc.w == 12345.f) out[0] = acc;
 }
 
-template <int U, int MODE>
+template <int U, int MODE, int ILV = 0>
 float run(const float4 *tab, const int *idx, int64_t n, int row_f4, float4 *out, int blocks) {
   cudaEvent_t a, b; CK(cudaEventCreate(&a)); CK(cudaEventCreate(&b));
-  replay<U, MODE><<<blocks, 256>>>(tab, idx, n, row_f4, out);
+  replay<U, MODE, ILV><<<blocks, 256>>>(tab, idx, n, row_f4, out);
   CK(cudaEventRecord(a));
   const int it = 10;
-  for (int i = 0; i < it; i++) replay<U, MODE><<<blocks, 256>>>(tab, idx, n, row_f4, out);
+  for (int i = 0; i < it; i++) replay<U, MODE, ILV><<<blocks, 256>>>(tab, idx, n, row_f4, out);
   CK(cudaEventRecord(b)); CK(cudaEventSynchronize(b));
   float ms; CK(cudaEventElapsedTime(&ms, a, b));
   return ms / it;
@@ -156,6 +170,10 @@ int main(int argc, char **argv) {
     printf("{\"blocks_per_sm\": %d, \"ms_u4\": %.4f, \"ms_u8\": %.4f, \"ms_u16\": %.4f, \"ms_u8_nol1\": %.4f, "
            "\"gbs_u8\": %.0f, \"gathers\": %lld}\n", occ, t4, t8, t16, t8n, bytes / (t8 * 1e-3) / 1e9, (long long)n);
   }
+  for (int occ : {2, 4, 8})
+    printf("{\"interleaved_blocks_per_sm\": %d, \"ms_u4\": %.4f, \"ms_u8\": %.4f}\n", occ,
+           run<4, 0, 1>(tab, idx, n, J / 4, out, sms * occ), run<8, 0, 1>(tab, idx, n, J / 4, out, sms * occ));
+  if (getenv("NO_TMA")) return 0;
   printf("{\"tma_r16_w8_b1\": %.4f, \"tma_r32_w4_b1\": %.4f, \"tma_r32_w6_b1\": %.4f, \"tma_r16_w4_b2\": %.4f, \"tma_r8_w8_b2\": %.4f}\n",
          run_tma<16, 8>(tab, idx, n, out, 1, sms), run_tma<32, 4>(tab, idx, n, out, 1, sms),
          run_tma<32, 6>(tab, idx, n, out, 1, sms), run_tma<16, 4>(tab, idx, n, out, 2, sms),
