@@ -868,12 +868,13 @@ cudaError_t run_csr_j(const lf_csr &A, const float *B, int64_t ldb, int J, float
 // CELL row is the whole C row, red.add otherwise (kRowRun rows pre-zeroed).
 constexpr int kGR = kGroupRows;  // CELL rows per group
 constexpr int kHT = 256;   // hash slots per warp (>= kGR * 32 distinct columns)
+constexpr int kGPad = 16;  // entry lists padded to a multiple of G * U (<= 16)
 struct GroupStage {
     int32_t key[kHT];      // column in hash slot, -1 = free
     int32_t idx_of[kHT];   // entry index of the slot's column
     int32_t hslot[kGR * 32];
-    int32_t ckey[kGR * 32];   // entry k: column ...
-    float4 cval[kGR * 32];    // ... and its value in each of the kGR rows (0 if absent)
+    const float *caddr[kGR * 32 + kGPad];  // entry k: its B row (resolved once) ...
+    float4 cval[kGR * 32 + kGPad];         // ... and its value in each of the kGR rows (0 if absent)
 };
 #ifndef LF_GROUP_MIN_BLOCKS
 #define LF_GROUP_MIN_BLOCKS 4
@@ -888,6 +889,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, LF_GROUP_MIN_BLOCKS) cell
     using VT = typename Cx::VT;
     using L = Layout<4, G, NV>;
     constexpr int U = 4;  // distinct columns in flight per lane group
+    static_assert(G * U <= kGPad, "entry padding");
     __shared__ __align__(16) GroupStage gs_all[kWarpsPerBlock];
     const int lane = threadIdx.x & 31;
     const int w = threadIdx.x >> 5;
@@ -946,27 +948,32 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, LF_GROUP_MIN_BLOCKS) cell
                 const int k = n_u + __popc(im & lt);
                 gs.idx_of[h] = k;
                 gs.hslot[k] = h;
-                gs.ckey[k] = c[r];
+                gs.caddr[k] = cx.rowaddr(c[r]);
                 gs.cval[k] = make_float4(0.f, 0.f, 0.f, 0.f);
             }
             n_u += __popc(im);
             __syncwarp();
             if (c[r] >= 0) atomicAdd(f4c(gs.cval[gs.idx_of[h]], r), v[r]);
         }
+        // pad the entry list to a multiple of G * U with zero entries (the
+        // zero row, values 0): the gather loop needs no bounds checks
+        const int n_pad = (n_u + G * U - 1) / (G * U) * (G * U);
+        if (lane < n_pad - n_u) {
+            gs.caddr[n_u + lane] = cx.rowaddr(-1);
+            gs.cval[n_u + lane] = make_float4(0.f, 0.f, 0.f, 0.f);
+        }
         __syncwarp();
         // gather each distinct B row once; lane group gi takes entries gi, gi + G, ...
         VT acc[kGR][NV];
 #pragma unroll
         for (int r = 0; r < kGR; r++) cx.zero(acc[r]);
-        for (int k0 = 0; k0 < n_u; k0 += G * U) {
+        for (int k0 = cx.g; k0 < n_pad; k0 += G * U) {
             VT b[U][NV];
             float4 vv[U];
 #pragma unroll
             for (int u = 0; u < U; u++) {
-                const int k = k0 + u * G + cx.g;
-                const bool ok = k < n_u;
-                vv[u] = ok ? gs.cval[k] : make_float4(0.f, 0.f, 0.f, 0.f);
-                cx.gather(cx.rowaddr(ok ? gs.ckey[k] : -1), b[u]);
+                vv[u] = gs.cval[k0 + u * G];
+                cx.gather(gs.caddr[k0 + u * G], b[u]);
             }
 #pragma unroll
             for (int u = 0; u < U; u++)

@@ -372,37 +372,6 @@ uint32_t mask_slots(int64_t n_cols) {
     return (uint32_t)m;
 }
 
-namespace {
-
-// Table 2 row-length statistics alone (P:L692-706): the features the
-// predictor needs BEFORE P is known (section 5.1-5.2), from row_ptr only
-// (8 B per row).  One thread per row, warp then block reduction, one set of
-// 64-bit atomics per block.  (Used when the statistics pass is too long to
-// run speculatively for P = 1, see lf_cell_configure.)
-__global__ void __launch_bounds__(kThreads) features_kernel(const int64_t *__restrict__ row_ptr, int64_t n_rows,
-                                                            StatsDev *st) {
-    unsigned long long mn = ~0ull, mx = 0, sum = 0, sq = 0;
-    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_rows; i += stride) {
-        const unsigned long long len = (unsigned long long)(__ldg(row_ptr + i + 1) - __ldg(row_ptr + i));
-        mn = min(mn, len);
-        mx = max(mx, len);
-        sum += len;
-        sq += len * len;
-    }
-    block_len_stats(mn, mx, sum, sq, st);
-}
-
-}  // namespace
-
-cudaError_t launch_features(const lf_csr &A, StatsDev *d_stats, cudaStream_t s) {
-    if (A.n_rows <= 0) return cudaSuccess;
-    const int64_t want = (A.n_rows + kThreads - 1) / kThreads;
-    const int grid = (int)std::min<int64_t>(want, (int64_t)num_sms() * 8);
-    features_kernel<<<grid, kThreads, 0, s>>>(A.row_ptr, A.n_rows, d_stats);
-    return cudaGetLastError();
-}
-
 // Grouped-path heuristic (cell_spmm.cu "grouped path"): on kGroupSamples
 // groups of kGroupRows consecutive rows spread evenly over A (rows of at most
 // 32 nonzeros; a group with a longer row is skipped), the number of DISTINCT
@@ -453,6 +422,39 @@ __global__ void __launch_bounds__(256) group_sample_kernel(const int64_t *__rest
         atomicAdd(&st->grp_union, (unsigned long long)n_u);
         atomicAdd(&st->grp_nnz, (unsigned long long)n_nz);
     }
+}
+
+namespace {
+
+// Table 2 row-length statistics alone (P:L692-706): the features the
+// predictor needs BEFORE P is known (section 5.1-5.2), from row_ptr only
+// (8 B per row).  One thread per row, warp then block reduction, one set of
+// 64-bit atomics per block.  (Used when the statistics pass is too long to
+// run speculatively for P = 1, see lf_cell_configure.)
+__global__ void __launch_bounds__(kThreads) features_kernel(const int64_t *__restrict__ row_ptr, int64_t n_rows,
+                                                            StatsDev *st) {
+    unsigned long long mn = ~0ull, mx = 0, sum = 0, sq = 0;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_rows; i += stride) {
+        const unsigned long long len = (unsigned long long)(__ldg(row_ptr + i + 1) - __ldg(row_ptr + i));
+        mn = min(mn, len);
+        mx = max(mx, len);
+        sum += len;
+        sq += len * len;
+    }
+    block_len_stats(mn, mx, sum, sq, st);
+}
+
+}  // namespace
+
+cudaError_t launch_features(const lf_csr &A, StatsDev *d_stats, cudaStream_t s) {
+    if (A.n_rows <= 0) return cudaSuccess;
+    const int64_t want = (A.n_rows + kThreads - 1) / kThreads;
+    const int grid = (int)std::min<int64_t>(want, (int64_t)num_sms() * 8);
+    features_kernel<<<grid, kThreads, 0, s>>>(A.row_ptr, A.n_rows, d_stats);
+    if (A.n_rows >= kGroupRows && A.nnz > 0)
+        group_sample_kernel<<<kGroupSamples / 8, 256, 0, s>>>(A.row_ptr, A.col_ind, A.n_rows, d_stats);
+    return cudaGetLastError();
 }
 
 cudaError_t launch_stats(const lf_csr &A, int P, StatsDev *d_stats, uint32_t *d_colmask, uint8_t *d_t0seg,

@@ -117,8 +117,21 @@ void table2_features(const lf_csr &A, int32_t J, const lf::StatsDev &st, double 
     f[7] = (double)J;
 }
 
-constexpr double kGroupedMaxRatio = 0.35;   // grouped path: distinct / nonzeros of 4-row groups
-constexpr double kGroupedMinMeanLen = 16.0; // ... and mean row length
+// Grouped SpMM path (cell_spmm.cu): worth it when consecutive rows share
+// many of their columns and the rows are long enough for a group to amortise
+// the column merge.  Measured on B200 (per-slot -> grouped ms, J = 64 / 128):
+// banded hw 4/8/12 (ratio 0.33-0.28) 1.06-1.8x faster, 32-wide dense blocks
+// (0.25) 1.8-2.0x, 27-point stencil (0.50) 1.2x; slower on R-MAT (0.96),
+// lognormal (~1), uniform (1.0, equal at J = 128) and rows of 8 (0.25, mean 8).
+constexpr double kGroupedMaxRatio = 0.6;    // distinct columns / nonzeros of 4-row groups
+constexpr double kGroupedMinMeanLen = 8.5;  // mean row length
+double group_ratio(const lf::StatsDev &st) {
+    return st.grp_nnz ? (double)st.grp_union / (double)st.grp_nnz : 1.0;
+}
+bool grouped_candidate(const lf::StatsDev &st, const lf_csr &A, int32_t J) {
+    const double mean = A.n_rows ? (double)st.len_sum / (double)A.n_rows : 0.0;
+    return J <= 128 && st.grp_nnz > 0 && group_ratio(st) <= kGroupedMaxRatio && mean >= kGroupedMinMeanLen;
+}
 
 // Algorithm 3 in exponent space (reading R8) over eq. 7 costs.
 int alg3(const int64_t *cost, int hi) {
@@ -226,6 +239,10 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
         int32_t pu = 1, pp = 1;
         if (lf_status st = lf_predict(f, max_parts, &pu, &pp)) return fail(st, "lf_predict");
         if (o.force_format == 0) use_cell = pu;
+        // the grouped CELL path (not in the paper's label space, trained on
+        // the per-slot kernel) beats the CSR kernel where it applies: keep
+        // CELL then (measured: 27-point stencil 0.82 vs 0.98 ms at J = 64)
+        if (o.force_format == 0 && !pu && grouped_candidate(*h_st, *A, J)) use_cell = 1;
         if (o.force_parts == 0 && pp != P) {
             P = pp;
             have = false;
@@ -292,13 +309,10 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
     // amortise the column merge (measured on B200: banded / dense-block rows
     // of 25-32 nonzeros at ratio <= 0.28 gain 1.3-1.45x, the 27-point stencil
     // at 0.50 and rows of 8 lose); needs every W_p <= 32 and J <= 128
-    cs.group_union_ratio = st.grp_nnz ? (double)st.grp_union / (double)st.grp_nnz : 1.0;
+    cs.group_union_ratio = group_ratio(st);
     bool narrow = true;
     for (int p = 0; p < P; p++) narrow = narrow && prm.max_width_log2[p] <= 5;
-    cs.spmm_grouped = (use_cell && narrow && J <= 128 && cs.group_union_ratio <= kGroupedMaxRatio &&
-                       cs.features[3] >= kGroupedMinMeanLen)
-                          ? 1
-                          : 0;
+    cs.spmm_grouped = (use_cell && narrow && grouped_candidate(st, *A, J)) ? 1 : 0;
     *out = prm;
     return LF_OK;
 }

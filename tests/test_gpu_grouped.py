@@ -107,12 +107,12 @@ def test_grouped_full_stencil_sampled(lf, grouped):
     assert np.all(np.abs(C[rows] - Cref) <= TOL * Cabs)
 
 
-@pytest.mark.parametrize("name,want", [("banded", 1), ("blockdiag32", 1), ("stencil", 0), ("rmat", 0),
+@pytest.mark.parametrize("name,want", [("banded", 1), ("blockdiag32", 1), ("stencil", 1), ("rmat", 0),
                                        ("blockdiag8", 0)])
 def test_grouped_heuristic(lf, monkeypatch, name, want):
     """lf_cell_configure's sampled group-union ratio picks the grouped path
-    where it measured faster (banded / 32-wide dense blocks), not on the
-    stencil, R-MAT or narrow rows; lf_spmm on the automatically chosen path
+    where it measured faster (banded, 32-wide dense blocks, 27-point stencil),
+    not on R-MAT or rows of 8; lf_spmm on the automatically chosen path
     matches the oracle."""
     monkeypatch.delenv("LF_GROUPED", raising=False)
     A_h = {"banded": lambda: gen.banded(20000, 12, seed=6), "blockdiag32": lambda: gen.blockdiag(16384, 32, seed=6),
