@@ -369,13 +369,20 @@ def main():
         return 0
     hbm_peak, peak_kind = peaks()
     P = params.n_parts
-    # configure: features_kernel + stats_rows/mark/cols; build: bucket_kernel<0>,
-    # tile_scan, bucket_kernel<1>, slot_fill, run_bounds (+ seg_kernel for P > 1);
-    # SpMM: zero_rows_kernel + cell_spmm_kernel (CSR format: csr_spmm_kernel only)
+    # configure (lf_api.cu): nnz <= 2^25 -> the statistics pass for P = 1 first
+    # (stats_rows, stats_mark, group_sample, stats_cols) and again if the
+    # predictor picks P > 1; larger -> features_kernel + group_sample first,
+    # then the statistics pass when CELL is used.  build: bucket_kernel<0>,
+    # tile_scan, pad_init, bucket_kernel<1>, slot_fill, run_bounds (+ seg_kernel
+    # for P > 1).  SpMM: zero_rows_kernel + cell_spmm (or grouped) kernel; the
+    # CSR format: csr_spmm_kernel only.
+    spec = args.parts != 0 or A_h.nnz <= (1 << 25)
+    cfg_launches = (4 + (4 if (params.n_parts != 1 and args.parts == 0 and params.use_cell) else 0)) if spec \
+        else (2 + (4 if params.use_cell else 0))
     if params.use_cell:
-        launches_per_step = 4 + 5 + (1 if P > 1 else 0) + 2
+        launches_per_step = cfg_launches + 6 + (1 if P > 1 else 0) + 2
     else:
-        launches_per_step = 4 + 1
+        launches_per_step = cfg_launches + 1
     sp_ms = ph["spmm"]
     line = {
         "metric": METRIC, "value": flops / (ms * 1e-3) / 1e9, "unit": "GFLOP/s", "n_gpus": world,

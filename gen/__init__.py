@@ -231,6 +231,9 @@ CONFIGS = {
     "c1_uniform1024": dict(J=32),
     "c2_rmat20": dict(J=128),
     "c3_stencil126": dict(J=64),
+    # configs[2] read literally ("banded FEM-like 2M rows, ~50M nnz"): a band
+    # of half-width 12 around the diagonal, 25 nonzeros per interior row
+    "c3b_banded2M": dict(J=64),
     "c4_reddit": dict(J=256),
 }
 
@@ -243,6 +246,8 @@ def config(name: str, seed: int = 0, kind: int = GRID, lo: int = -3, hi: int = 3
         m = rmat(20, 16, seed=seed, kind=kind, lo=lo, hi=hi)
     elif name == "c3_stencil126":
         m = stencil27(126, seed, kind, lo, hi)
+    elif name == "c3b_banded2M":
+        m = banded(2_000_000, 12, seed=seed, kind=kind, lo=lo, hi=hi)
     elif name == "c4_reddit":
         m = powerlaw(232965, 114615892, 1.2, seed, kind, lo, hi)
     else:

@@ -17,3 +17,7 @@ if [ -z "$SKIP_NCU" ]; then
      -f -o gpurun_out/${TAG}_spmm_full python scripts/prof.py c2_rmat20 4 > gpurun_out/${TAG}_ncu.log 2>&1
 fi
 tail -3 gpurun_out/${TAG}_smoke.txt; tail -3 gpurun_out/${TAG}_pytest_gpu.txt 2>/dev/null; cat gpurun_out/${TAG}_bench.json
+# per-config SpMM timing (configure / build / spmm phases; grouped path where chosen)
+for c in c1_uniform1024 c3_stencil126 c3b_banded2M c4_reddit; do
+  echo "$c $(timeout 300 python scripts/spmm_time.py $c iters=10 | tail -1)" >> gpurun_out/${TAG}_configs.txt
+done

@@ -90,3 +90,15 @@ def test_random_small_edge_cases():
     _check_csr(m, dedup=False)
     assert (m.row_lengths() == 0).any()
     assert (m.val == 0).any()
+
+
+def test_banded_config_closed_form():
+    """c3b_banded2M (BASELINE configs[2] read literally): half-width 12 band on
+    2,000,000 rows -> 25 n - 2 (1 + ... + 12) nonzeros, columns i-12..i+12."""
+    A, J = gen.config("c3b_banded2M")
+    n = 2_000_000
+    assert (A.n_rows, A.n_cols, J) == (n, n, 64)
+    assert A.nnz == 25 * n - 2 * 78
+    rp, ci = np.asarray(A.row_ptr), np.asarray(A.col_ind)
+    for i in (0, 5, 12, 999_999, n - 13, n - 1):
+        assert np.array_equal(ci[rp[i]:rp[i + 1]], np.arange(max(i - 12, 0), min(i + 12, n - 1) + 1))

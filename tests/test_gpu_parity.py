@@ -230,7 +230,7 @@ def test_row_shard_view(lf):
 
 
 # ---- full-size BASELINE configs, the bench's launch configuration ----------
-FULL = ["c1_uniform1024", "c2_rmat20", "c3_stencil126"]
+FULL = ["c1_uniform1024", "c2_rmat20", "c3_stencil126", "c3b_banded2M"]
 
 
 @pytest.mark.parametrize("name", FULL)
