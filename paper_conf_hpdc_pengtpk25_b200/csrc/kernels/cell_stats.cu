@@ -79,8 +79,8 @@ __device__ __forceinline__ void block_len_stats(unsigned long long mn, unsigned 
 #define LF_MARK_TILE 4096
 #endif
 constexpr int kMarkTile = LF_MARK_TILE;
-#ifndef LF_MARK_MATCH
-#define LF_MARK_MATCH 0
+#ifndef LF_MARK_MIN_BLOCKS
+#define LF_MARK_MIN_BLOCKS 4
 #endif  // nonzeros per block of the marking pass
 
 __global__ void __launch_bounds__(kThreads) stats_rows_kernel(const int64_t *__restrict__ row_ptr,
@@ -162,8 +162,11 @@ __global__ void __launch_bounds__(kThreads) stats_rows_kernel(const int64_t *__r
 #define LF_MARK_HASH 1
 #endif
 #ifndef LF_MARK_MODE
-#define LF_MARK_MODE 1  // 0: L2 check then RED; 1: RED only (measured fastest, c2: 107 vs 120 us); 2: L1-cached check
+#define LF_MARK_MODE 3  // tiles of one natural bucket: 3 = block smem filter, then one RED per column;
+                        // other tiles: 0 = L2 check then RED, 2 = L1-cached check, 1 / 3 = RED only
 #endif
+constexpr int kMarkFilter = 2048;            // direct-mapped (column, bits) slots per block (mode 3)
+constexpr uint32_t kFilterEmpty = 0xFFFFFFFFu;
 constexpr uint32_t kHashOdd = LF_MARK_HASH ? 0x9E3779B1u : 1u;
 __device__ __forceinline__ uint32_t hslot(int32_t c, uint32_t kmask) { return ((uint32_t)c * kHashOdd) & kmask; }
 __device__ __forceinline__ uint32_t ld_ca(const uint32_t *p) {
@@ -172,7 +175,7 @@ __device__ __forceinline__ uint32_t ld_ca(const uint32_t *p) {
     return v;
 }
 
-__global__ void __launch_bounds__(kThreads, 4) stats_mark_kernel(const int64_t *__restrict__ row_ptr,
+__global__ void __launch_bounds__(kThreads, LF_MARK_MIN_BLOCKS) stats_mark_kernel(const int64_t *__restrict__ row_ptr,
                                                               const int32_t *__restrict__ col, int64_t n_rows,
                                                               int64_t S, int P,
                                                               const uint8_t *__restrict__ t0seg,
@@ -182,9 +185,19 @@ __global__ void __launch_bounds__(kThreads, 4) stats_mark_kernel(const int64_t *
     __shared__ int32_t cnt[kMarkTile];     // rows starting at a tile position -> inclusive scan
     __shared__ uint8_t rt0[kMarkTile + 1]; // t0 of the tile's rows (P == 1)
     __shared__ int32_t wsum[kThreads / 32];
+    __shared__ uint32_t fkey[kMarkFilter], fbits[kMarkFilter];  // block filter of uniform tiles
+    for (int q = threadIdx.x; q < kMarkFilter; q += blockDim.x) {
+        fkey[q] = kFilterEmpty;
+        fbits[q] = 0u;
+    }
     constexpr int K = kMarkTile / kThreads;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    __shared__ unsigned s_tmin, s_tmax;  // natural buckets of the tile's non-empty rows (P == 1)
     for (int q = threadIdx.x; q < kMarkTile; q += blockDim.x) cnt[q] = 0;
+    if (threadIdx.x == 0) {
+        s_tmin = 0xFFFFFFFFu;
+        s_tmax = 0u;
+    }
     const int64_t base = row_ptr[0];
     const int64_t T = blockIdx.x;
     const int64_t rlo = tile_row[T];
@@ -193,6 +206,7 @@ __global__ void __launch_bounds__(kThreads, 4) stats_mark_kernel(const int64_t *
     const int64_t qb = T + 1 < n_tiles ? base + tile_pos[T + 1] : row_ptr[n_rows];
     __syncthreads();
     {
+        unsigned lmin = 0xFFFFFFFFu, lmax = 0u;
         constexpr int RU = 8;  // independent row_ptr loads in flight per thread
         for (int64_t r0 = rlo + threadIdx.x; r0 <= rhi; r0 += (int64_t)blockDim.x * RU) {
             int64_t sr[RU], er[RU];
@@ -206,13 +220,29 @@ __global__ void __launch_bounds__(kThreads, 4) stats_mark_kernel(const int64_t *
             for (int u = 0; u < RU; u++) {
                 const int64_t r = r0 + (int64_t)u * blockDim.x;
                 if (r > rhi) break;
-                if (P == 1) rt0[r - rlo] = (uint8_t)ceil_log2_i64(max(er[u] - sr[u], (int64_t)1));
+                if (P == 1) {
+                    const unsigned t0 = (unsigned)ceil_log2_i64(max(er[u] - sr[u], (int64_t)1));
+                    rt0[r - rlo] = (uint8_t)t0;
+                    if (er[u] > sr[u]) {
+                        lmin = min(lmin, t0);
+                        lmax = max(lmax, t0);
+                    }
+                }
                 if (r > rlo && sr[u] < qb - qa) atomicAdd(&cnt[sr[u]], 1);
             }
         }
+        lmin = __reduce_min_sync(kFull, lmin);
+        lmax = __reduce_max_sync(kFull, lmax);
+        if (lane == 0 && P == 1) {
+            atomicMin(&s_tmin, lmin);
+            atomicMax(&s_tmax, lmax);
+        }
     }
     __syncthreads();
-    {  // inclusive scan of cnt, conflict-free: warp w scans its 512 entries in
+    // every non-empty row of the tile in one natural bucket (banded, stencil,
+    // regular rows): every nonzero gets that bit, no position -> row scan
+    const bool uni = P == 1 && s_tmin == s_tmax;
+    if (!uni) {  // inclusive scan of cnt, conflict-free: warp w scans its 512 entries in
        // 32-wide chunks (shuffles), then adds the totals of the warps before it
         constexpr int PER_WARP = kMarkTile / (kThreads / 32);
         int32_t carry = 0;
@@ -245,30 +275,58 @@ __global__ void __launch_bounds__(kThreads, 4) stats_mark_kernel(const int64_t *
     for (int k = 0; k < K; k++) {
         bit[k] = 0;
         if (c[k] < 0) continue;
+        if (uni) {
+            bit[k] = 1u << s_tmin;
+            continue;
+        }
         const int rr = cnt[k * kThreads + threadIdx.x];
         if (P == 1) bit[k] = 1u << rt0[rr];
         else bit[k] = 1u << __ldg(t0seg + (rlo + rr) * P + (int)(c[k] / S));
     }
-    // One RED per (column, bit) (LF_MARK_MODE 1).  Reading the mask word
-    // first and skipping bits already set (mode 0) issues as many L2
-    // requests and adds a dependent load: measured slower on B200.
-    uint32_t h[K], have[K];
+    uint32_t h[K];
 #pragma unroll
-    for (int k = 0; k < K; k++) {
-#if LF_MARK_MATCH
-        const unsigned long long key = ((unsigned long long)(uint32_t)c[k] << 32) | bit[k];
-        const unsigned peers = __match_any_sync(kFull, key);
-        const bool leader = c[k] >= 0 && (peers & ((1u << lane) - 1u)) == 0;
-        bit[k] = leader ? bit[k] : 0u;
-#endif
-        h[k] = c[k] >= 0 ? hslot(c[k], kmask) : 0u;
+    for (int k = 0; k < K; k++) h[k] = c[k] >= 0 ? hslot(c[k], kmask) : 0u;
+    if (LF_MARK_MODE == 3 && uni) {
+        // block-level merge (tiles of one natural bucket: banded / stencil
+        // rows, where a tile of ~4096 nonzeros covers ~200 distinct columns):
+        // (column, bits) pairs collect in a direct-mapped shared-memory filter
+        // (slot = low bits of the column's hashed slot; read first, most are
+        // hits); a column colliding with another goes to L2 at once; after
+        // the tile every filled slot issues ONE RED.
+#pragma unroll
+        for (int k = 0; k < K; k++) {
+            if (c[k] < 0) continue;
+            const int f = (int)(h[k] & (kMarkFilter - 1));
+            uint32_t cur = reinterpret_cast<volatile uint32_t *>(fkey)[f];
+            if (cur == kFilterEmpty) {
+                cur = atomicCAS(&fkey[f], kFilterEmpty, (uint32_t)c[k]);
+                if (cur == kFilterEmpty) cur = (uint32_t)c[k];
+            }
+            if (cur == (uint32_t)c[k]) {
+                if ((reinterpret_cast<volatile uint32_t *>(fbits)[f] & bit[k]) != bit[k]) atomicOr(&fbits[f], bit[k]);
+            } else {
+                atomicOr(mask + h[k], bit[k]);  // slot taken by another column
+            }
+        }
+        __syncthreads();
+        for (int f = threadIdx.x; f < kMarkFilter; f += blockDim.x) {
+            const uint32_t key = fkey[f];
+            if (key != kFilterEmpty) atomicOr(mask + hslot((int32_t)key, kmask), fbits[f]);
+        }
+        return;
     }
+    // other tiles: one RED per (column, bit) (LF_MARK_MODE 1 everywhere).
+    // Reading the mask word first and skipping bits already set (mode 0)
+    // issues as many L2 requests and adds a dependent load: slower on B200.
+    {
+        uint32_t have[K];
 #pragma unroll
-    for (int k = 0; k < K; k++)
-        have[k] = LF_MARK_MODE == 1 ? 0u : LF_MARK_MODE == 2 ? ld_ca(mask + h[k]) : __ldcg(mask + h[k]);
+        for (int k = 0; k < K; k++)
+            have[k] = LF_MARK_MODE == 0 ? __ldcg(mask + h[k]) : LF_MARK_MODE == 2 ? ld_ca(mask + h[k]) : 0u;
 #pragma unroll
-    for (int k = 0; k < K; k++)
-        if ((have[k] & bit[k]) != bit[k]) atomicOr(mask + h[k], bit[k]);
+        for (int k = 0; k < K; k++)
+            if (c[k] >= 0 && (have[k] & bit[k]) != bit[k]) atomicOr(mask + h[k], bit[k]);
+    }
 }
 
 // Pass 3 -- one thread per mask SLOT (coalesced loads; the column is the
