@@ -58,6 +58,12 @@ __device__ __forceinline__ void segment_of(const int64_t *__restrict__ row_ptr, 
 }
 
 // PASS 0: count (tile totals + per-row CELL-row counts); PASS 1: place.
+// A row folded into more than kThreadSubRows CELL rows has its sub-rows
+// written by the whole warp (coalesced) instead of by its own thread.
+#ifndef LF_THREAD_SUBROWS
+#define LF_THREAD_SUBROWS 32
+#endif
+constexpr int kThreadSubRows = LF_THREAD_SUBROWS;
 template <int PASS>
 __global__ void __launch_bounds__(kThreads)
     bucket_kernel(const int64_t *__restrict__ row_ptr, const int32_t *__restrict__ seg_rel, int64_t n_rows, int P,
@@ -128,7 +134,7 @@ __global__ void __launch_bounds__(kThreads)
             row_mode[i] = kRowEmpty;  // (P > 1: pre-filled, another partition may own the row)
         }
         const int64_t W = int64_t(1) << (key == kNoKey ? 0 : key);
-        if (n_sub <= 32) {
+        if (n_sub <= kThreadSubRows) {
             for (int64_t s = 0; s < n_sub; s++) {
                 row_ind[pos + s] = (int32_t)i;
                 row_tag[pos + s] = tag | (s == 0 ? 2 : 0) | (s == n_sub - 1 ? 1 : 0);
@@ -137,7 +143,7 @@ __global__ void __launch_bounds__(kThreads)
             }
         }
         // long folded rows: the warp writes their sub-rows together
-        unsigned long_lanes = __ballot_sync(0xffffffffu, n_sub > 32);
+        unsigned long_lanes = __ballot_sync(0xffffffffu, n_sub > kThreadSubRows);
         while (long_lanes) {
             const int src = __ffs(long_lanes) - 1;
             long_lanes &= long_lanes - 1;
