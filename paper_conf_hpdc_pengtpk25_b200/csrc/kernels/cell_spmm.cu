@@ -1035,6 +1035,263 @@ cudaError_t run_grouped_j(const SpmmArgs &a, cudaStream_t s) {
     return a.J == Layout<4, G, NV>::JT ? run_grouped<G, NV, true>(a, s) : run_grouped<G, NV, false>(a, s);
 }
 
+// ---- tensor-core grouped path (mma.sync m16n8k8 TF32, 3xTF32 split) -------
+// A group of kMR = 16 consecutive CELL rows of a bucket (W <= 32) is one dense
+// contraction: C_group[16 x J] = V[16 x K] . Bg[K x J], K = the group's
+// distinct columns (entries) and Bg their B rows.  On banded / dense-block
+// matrices K is small (band half-width 12: K = 40 for 16 rows of 25), so
+// every B row is gathered about K / 16 = 2.5 times per row of A instead of 25.
+// The warp merges the rows' columns in a shared-memory hash set (as the
+// grouped path) and scatters the values into V (smem, zero where a row lacks
+// the column), then runs the contraction on the tensor cores with fp32
+// accuracy from three TF32 products (a_hi b_hi + a_hi b_lo + a_lo b_hi, each
+// operand x = hi + lo with hi = tf32(x)); integer-valued inputs are exact.
+// Fragment mapping: n-tile j, fragment column n of lane group g = lane / 4
+// is C column g * NT + j for B and (2t or 2t+1) * NT + j for D (t = lane % 4),
+// so each lane loads NT contiguous floats of a B row (NT / 4 LDG.128) and
+// owns 2 NT contiguous floats of its two C rows (g, g + 8).  A group whose K
+// exceeds kKCap is computed by the plain per-slot loop instead.
+constexpr int kMR = 16;           // rows per tensor-core group (MMA M)
+constexpr int kKCap = 64;         // max distinct columns per group
+constexpr int kMHT = 128;         // hash slots (<= kKCap + 32 keys ever inserted)
+constexpr int kVStride = kKCap + 4;  // V row stride (floats): conflict-free A-fragment loads
+constexpr int kMmaWarps = 4;
+struct MmaStage {
+    int32_t key[kMHT];
+    int32_t idx_of[kMHT];
+    int32_t hslot[kKCap + 32];
+    const float *caddr[kKCap + 8];
+    float V[kMR * kVStride];
+};
+
+__device__ __forceinline__ uint32_t tf32_hi(float x) {
+    uint32_t r;
+    asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));
+    return r;
+}
+__device__ __forceinline__ void split_tf32(float x, uint32_t &hi, uint32_t &lo) {
+    hi = tf32_hi(x);
+    lo = tf32_hi(x - __uint_as_float(hi));
+}
+__device__ __forceinline__ void mma_tf32(float (&d)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) {
+    asm volatile(
+        "mma.sync.aligned.m16n8k8.row.col.f32.tf32.tf32.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
+        "{%0,%1,%2,%3};"
+        : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3])
+        : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
+}
+
+template <int NT>
+__global__ void __launch_bounds__(kMmaWarps * 32) cell_spmm_mma_kernel(const SpmmArgs a) {
+    const int J = a.J;  // a multiple of 8 NT
+    __shared__ __align__(16) MmaStage ms_all[kMmaWarps];
+    const int lane = threadIdx.x & 31;
+    const int w = threadIdx.x >> 5;
+    MmaStage &ms = ms_all[w];
+    for (int q = lane; q < kMHT; q += 32) ms.key[q] = -1;
+    __syncwarp();
+    const uint64_t pol = policy_evict_first();
+    const int64_t nw = (int64_t)gridDim.x * kMmaWarps;
+    zero_rows_warp(a.row_mode, a.n_rows, a.C, a.ldc, a.J, true, 1u << kRowEmpty,
+                   (int64_t)blockIdx.x * kMmaWarps + w, nw, lane, pol);
+    const unsigned lt = (1u << lane) - 1u;
+    const int g = lane >> 2, t = lane & 3;
+    const float *zrow = reinterpret_cast<const float *>(g_zero_row);
+    const int64_t n = a.n_groups_m;
+    int bcur = 0;
+    int sz = claim_size(n, 0, nw);
+    int64_t grp = claim_get(claim_issue(a.ctr + 1, sz, lane));
+    int64_t gend = min(grp + sz, n);
+    while (grp < n) {
+        while (bcur + 1 < a.nb_g && __ldg(&a.bk_m[bcur + 1].task_off) <= grp) bcur++;
+        const BucketDev *bk = a.bk_m + bcur;
+        const int W = 1 << __ldg(&bk->t);
+        const int64_t r0 = (grp - __ldg(&bk->task_off)) * kMR;
+        const int nr = (int)min((int64_t)kMR, __ldg(&bk->n_rows_pad) - r0);
+        const int64_t row0 = __ldg(&bk->row_off) + r0;
+        const int64_t slot0 = __ldg(&bk->slot_off) + r0 * W;
+        const int32_t tag_l = lane < nr ? __ldg(a.row_tag + row0 + lane) : -1;
+        for (int q = lane; q < kMR * kVStride / 4; q += 32)
+            reinterpret_cast<float4 *>(ms.V)[q] = make_float4(0.f, 0.f, 0.f, 0.f);
+        // merge the rows' columns (rows in order, lanes in order: entries numbered
+        // deterministically); V[r][entry] += value
+        int n_u = 0;
+        bool over = false;
+        int32_t cr[kMR];
+        float vr[kMR];
+#pragma unroll
+        for (int r = 0; r < kMR; r++) {  // all the group's slots in flight at once
+            const bool in = r < nr && lane < W;
+            cr[r] = in ? ld_stream(a.col + slot0 + (int64_t)r * W + lane, pol) : -1;
+            vr[r] = in ? ld_stream(a.val + slot0 + (int64_t)r * W + lane, pol) : 0.f;
+        }
+#pragma unroll
+        for (int r = 0; r < kMR; r++) {
+            if (over) break;
+            const int32_t c = cr[r];
+            const float v = vr[r];
+            bool need = c >= 0, ins = false;
+            int h = (int)(((uint32_t)c * 0x9E3779B1u) >> 25);  // 7 bits: kMHT = 128
+            while (__any_sync(kFull, need)) {
+                if (need) {
+                    const int prev = atomicCAS(&ms.key[h], -1, c);
+                    if (prev == -1) ins = true;
+                    if (prev == -1 || prev == c) need = false;
+                    else h = (h + 1) & (kMHT - 1);
+                }
+            }
+            const unsigned im = __ballot_sync(kFull, ins);
+            if (ins) {
+                const int k = n_u + __popc(im & lt);
+                ms.idx_of[h] = k;
+                ms.hslot[k] = h;
+                ms.caddr[k] = k < kKCap ? a.B + (int64_t)c * a.ldb : zrow;
+            }
+            n_u += __popc(im);
+            __syncwarp();
+            over = n_u > kKCap;
+            if (!over && c >= 0) atomicAdd(&ms.V[r * kVStride + ms.idx_of[h]], v);
+        }
+        __syncwarp();
+        if (!over) {
+            const int n_pad = (n_u + 7) & ~7;
+            if (lane < n_pad - n_u) ms.caddr[n_u + lane] = zrow;
+            __syncwarp();
+            // J in slices of 8 NT columns; per slice the k-steps run with the
+            // next step's B rows loaded before this step's products
+            for (int jp = 0; jp < a.J; jp += 8 * NT) {
+                float acc[NT][4];
+#pragma unroll
+                for (int j = 0; j < NT; j++) acc[j][0] = acc[j][1] = acc[j][2] = acc[j][3] = 0.f;
+                float b0[NT], b1[NT], n0[NT], n1[NT];
+                auto load_b = [&](int k0, float (&x0)[NT], float (&x1)[NT]) {
+                    const float *e0 = ms.caddr[k0 + t], *e1 = ms.caddr[k0 + t + 4];
+                    const bool z0 = e0 == zrow, z1 = e1 == zrow;
+#pragma unroll
+                    for (int q = 0; q < NT; q += 4) {
+                        const float4 y0 = z0 ? make_float4(0.f, 0.f, 0.f, 0.f)
+                                             : __ldg(reinterpret_cast<const float4 *>(e0 + jp + g * NT + q));
+                        const float4 y1 = z1 ? make_float4(0.f, 0.f, 0.f, 0.f)
+                                             : __ldg(reinterpret_cast<const float4 *>(e1 + jp + g * NT + q));
+                        x0[q] = y0.x, x0[q + 1] = y0.y, x0[q + 2] = y0.z, x0[q + 3] = y0.w;
+                        x1[q] = y1.x, x1[q + 1] = y1.y, x1[q + 2] = y1.z, x1[q + 3] = y1.w;
+                    }
+                };
+                if (n_pad > 0) load_b(0, n0, n1);
+                for (int k0 = 0; k0 < n_pad; k0 += 8) {
+#pragma unroll
+                    for (int j = 0; j < NT; j++) {
+                        b0[j] = n0[j];
+                        b1[j] = n1[j];
+                    }
+                    if (k0 + 8 < n_pad) load_b(k0 + 8, n0, n1);
+                    uint32_t ah[4], al[4];
+                    split_tf32(ms.V[g * kVStride + k0 + t], ah[0], al[0]);
+                    split_tf32(ms.V[(g + 8) * kVStride + k0 + t], ah[1], al[1]);
+                    split_tf32(ms.V[g * kVStride + k0 + t + 4], ah[2], al[2]);
+                    split_tf32(ms.V[(g + 8) * kVStride + k0 + t + 4], ah[3], al[3]);
+#pragma unroll
+                    for (int j = 0; j < NT; j++) {
+                        uint32_t bh0, bl0, bh1, bl1;
+                        split_tf32(b0[j], bh0, bl0);
+                        split_tf32(b1[j], bh1, bl1);
+                        mma_tf32(acc[j], al, bh0, bh1);
+                        mma_tf32(acc[j], ah, bl0, bl1);
+                        mma_tf32(acc[j], ah, bh0, bh1);
+                    }
+                }
+                // rows g and g + 8: columns jp + [2t NT, 2t NT + 2 NT)
+#pragma unroll
+                for (int half = 0; half < 2; half++) {
+                    const int r = g + 8 * half;
+                    const int32_t tag = __shfl_sync(kFull, tag_l, r);
+                    if (r < nr && tag >= 0) {
+                        float *p = a.C + (int64_t)tag_row(tag) * a.ldc + jp + 2 * t * NT;
+                        const bool plain = tag_whole(tag);
+#pragma unroll
+                        for (int q = 0; q < NT; q += 4) {
+                            const float4 lo4 = make_float4(acc[q][2 * half], acc[q + 1][2 * half],
+                                                           acc[q + 2][2 * half], acc[q + 3][2 * half]);
+                            const float4 hi4 = make_float4(acc[q][2 * half + 1], acc[q + 1][2 * half + 1],
+                                                           acc[q + 2][2 * half + 1], acc[q + 3][2 * half + 1]);
+                            if (plain) {
+                                Vec<4>::store(p + q, lo4, pol);
+                                Vec<4>::store(p + NT + q, hi4, pol);
+                            } else {
+                                Vec<4>::red(p + q, lo4);
+                                Vec<4>::red(p + NT + q, hi4);
+                            }
+                        }
+                    }
+                }
+            }
+        } else {
+            // too many distinct columns: the rows one by one, per slot (lane
+            // covers 4 of the J columns; J = 8 NT <= 128)
+            for (int r = 0; r < nr; r++) {
+                const int32_t tag = __shfl_sync(kFull, tag_l, r);
+                if (tag < 0) continue;
+                const int32_t c = lane < W ? ld_stream(a.col + slot0 + (int64_t)r * W + lane, pol) : -1;
+                const float v = lane < W ? ld_stream(a.val + slot0 + (int64_t)r * W + lane, pol) : 0.f;
+                float4 s = make_float4(0.f, 0.f, 0.f, 0.f);
+                for (int q = 0; q < W; q++) {
+                    const int32_t cq = __shfl_sync(kFull, c, q);
+                    const float vq = __shfl_sync(kFull, v, q);
+                    if (cq < 0 || 4 * lane >= J) continue;
+                    Vec<4>::fma(s, vq, __ldg(reinterpret_cast<const float4 *>(a.B + (int64_t)cq * a.ldb) + lane));
+                }
+                if (4 * lane < J) {
+                    float *p = a.C + (int64_t)tag_row(tag) * a.ldc + 4 * lane;
+                    if (tag_whole(tag)) Vec<4>::store(p, s, pol);
+                    else Vec<4>::red(p, s);
+                }
+            }
+        }
+        for (int k = lane; k < n_u; k += 32) ms.key[ms.hslot[k]] = -1;  // free the used slots
+        __syncwarp();
+        if (++grp >= gend) {
+            sz = claim_size(n, grp, nw);
+            grp = claim_get(claim_issue(a.ctr + 1, sz, lane));
+            gend = min(grp + sz, n);
+        }
+    }
+    if (lane == 0) {  // the last warp out resets the queue counters (as cell_spmm_kernel)
+        __threadfence();
+        if (atomicAdd(a.ctr + 2, 1ull) == (unsigned long long)gridDim.x * kMmaWarps - 1) {
+            __threadfence();
+            a.ctr[0] = 0;
+            a.ctr[1] = 0;
+            a.ctr[2] = 0;
+        }
+    }
+}
+
+template <int NT>
+cudaError_t run_mma(const SpmmArgs &a, cudaStream_t s) {
+    static int cap = 0;
+    auto fn = cell_spmm_mma_kernel<NT>;
+    if (!cap) {
+        int occ = 0, sms = 0, dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kMmaWarps * 32, 0);
+        cap = std::max(1, occ) * std::max(1, sms);
+    }
+    const int64_t want = std::max<int64_t>((a.n_groups_m + kMmaWarps - 1) / kMmaWarps,
+                                           (a.n_rows + 32 * kMmaWarps - 1) / (32 * kMmaWarps));
+    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(cap, want));
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3((unsigned)grid);
+    cfg.blockDim = dim3(kMmaWarps * 32);
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, fn, a);
+}
+
 bool vec4_ok(const float *B, int64_t ldb, const float *C, int64_t ldc, int J) {
     return J % 4 == 0 && ldb % 4 == 0 && ldc % 4 == 0 && ((uintptr_t)B & 15) == 0 && ((uintptr_t)C & 15) == 0;
 }
@@ -1057,9 +1314,18 @@ bool grouped_ok(const SpmmArgs &a) {
     return a.grouped && a.nb_g > 0 && vec4_ok(a.B, a.ldb, a.C, a.ldc, a.J) && a.J <= 128;
 }
 
+bool mma_ok(const SpmmArgs &a) {
+    return a.mma && a.nb_g > 0 && vec4_ok(a.B, a.ldb, a.C, a.ldc, a.J) && a.J % 64 == 0 && a.J <= 128;
+}
+
 cudaError_t launch_cell_spmm(const SpmmArgs &a, cudaStream_t s) {
     if (a.J == 0 || a.n_rows == 0) return cudaSuccess;
     const bool v4 = vec4_ok(a.B, a.ldb, a.C, a.ldc, a.J);
+    if (mma_ok(a)) {
+        cudaError_t e = zero_red_rows(a, true, s);
+        if (e != cudaSuccess) return e;
+        return run_mma<8>(a, s);
+    }
     if (grouped_ok(a)) {  // runs of folded rows are split across groups: red.add, pre-zeroed
         cudaError_t e = zero_red_rows(a, true, s);
         if (e != cudaSuccess) return e;

@@ -437,6 +437,12 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
                 h->n_groups += (d.n_rows_pad + lf::kGroupRows - 1) / lf::kGroupRows;
                 h->h_buckets.push_back(d);
             }
+            for (int q = 0; q < nb_all; q++) {  // and again for 16-row groups (tensor-core path)
+                lf::BucketDev d = h->h_buckets[q];
+                d.task_off = h->n_groups_m;
+                h->n_groups_m += (d.n_rows_pad + 15) / 16;
+                h->h_buckets.push_back(d);
+            }
             h->nb_g = nb_all;
         }
         if (h->buckets.size() > 2048) return fail(LF_ERR_UNSUPPORTED, "more than 2048 buckets");
@@ -563,8 +569,10 @@ lf_status lf_spmm(const lf_cell *h, const float *B, int64_t ldb, int32_t J, floa
                    h->ctr_ring + 4 * (h->launch_seq.fetch_add(1, std::memory_order_relaxed) % kCtrSlots), h->col_ind, h->val,
                    h->row_tag,
                    B, ldb, C, ldc, J,
-                   h->d_buckets + nb + h->nb_n + h->nb_w, h->nb_g, h->grouped, h->n_groups};
+                   h->d_buckets + nb + h->nb_n + h->nb_w, h->nb_g, h->grouped, h->n_groups,
+                   h->d_buckets + nb + h->nb_n + h->nb_w + h->nb_g, h->mma, h->n_groups_m};
     if (const char *g = std::getenv("LF_GROUPED")) a.grouped = g[0] == '1';
+    if (const char *g = std::getenv("LF_MMA")) a.mma = g[0] == '1';
     LF_CUDA(lf::launch_cell_spmm(a, s));
     return LF_OK;
 }

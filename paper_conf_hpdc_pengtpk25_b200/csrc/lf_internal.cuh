@@ -146,6 +146,10 @@ struct SpmmArgs {
     int nb_g;
     int grouped;  // use it (when J and the alignment allow)
     int64_t n_groups;
+    // tensor-core grouped path: the same buckets, task_off counting 16-row groups
+    const BucketDev *bk_m;
+    int mma;
+    int64_t n_groups_m;
 };
 cudaError_t launch_cell_spmm(const SpmmArgs &a, cudaStream_t s);  // pre-zeroes kRowRed rows itself
 cudaError_t launch_csr_spmm(const lf_csr &A, const float *B, int64_t ldb, int J, float *C, int64_t ldc,
@@ -171,6 +175,8 @@ struct lf_cell {
     int nb_g = 0;            // grouped-path buckets (= nb when every W <= 32, else 0)
     int64_t n_groups = 0;
     int grouped = 0;         // lf_spmm takes the grouped path
+    int64_t n_groups_m = 0;  // 16-row groups (tensor-core grouped path)
+    int mma = 0;             // lf_spmm takes the tensor-core grouped path
     // work-queue counters, kCtrSlots slots of 4 (wide, narrow, warps done, -)
     // in the pool: launch k uses slot k % kCtrSlots and its last warp resets
     // it, so lf_spmm needs no allocation or memset per call

@@ -1,6 +1,6 @@
 """GPU parity of the grouped (column-merged) SpMM path against the oracle.
 
-The grouped path (cell_spmm.cu) applies when every
+The grouped paths (cell_spmm.cu) apply when every
 bucket has W <= 32, B / C are 16-byte aligned and J <= 256: kGroupRows
 consecutive CELL rows share one gather per distinct column.  It must give the
 same C as Algorithm 1: exactly on integer inputs (any atomic / summation
@@ -25,9 +25,15 @@ def lf():
     return m
 
 
-@pytest.fixture
-def grouped(monkeypatch):
-    monkeypatch.setenv("LF_GROUPED", "1")
+@pytest.fixture(params=["LF_GROUPED", "LF_MMA"])
+def grouped(request, monkeypatch):
+    """Both grouped paths: the CUDA-core one (LF_GROUPED) and the tensor-core
+    one (LF_MMA: 16-row groups, 3xTF32 mma.sync; J in {64, 128}, otherwise
+    the launch falls back to the per-slot path)."""
+    monkeypatch.setenv("LF_GROUPED", "0")
+    monkeypatch.setenv("LF_MMA", "0")
+    monkeypatch.setenv(request.param, "1")
+    return request.param
 
 
 def run(lf, A_h, B_h, P, e, k=None):
@@ -77,17 +83,22 @@ def test_grouped_banded_float(lf, grouped, hw, e):
     assert np.all(np.abs(C - Cref) <= TOL * Cabs)
 
 
-def test_grouped_equals_per_slot_path(lf, monkeypatch):
-    """Same handle, both paths: equal on integer inputs; repeated grouped
-    launches (queue counters reset by the last warp) stay equal."""
+@pytest.mark.parametrize("env", ["LF_GROUPED", "LF_MMA"])
+@pytest.mark.parametrize("J", [64, 128])
+def test_grouped_equals_per_slot_path(lf, monkeypatch, env, J):
+    """Same handle, per-slot vs grouped path: equal on integer inputs (R-MAT:
+    most 16-row groups exceed the tensor-core path's 64 distinct columns and
+    take its per-row fallback); repeated launches (queue counters reset by
+    the last warp) stay equal."""
     A_h = gen.rmat(12, 16, seed=5, kind=gen.INT, lo=-3, hi=3)
-    B_h = gen.dense(A_h.n_cols, 128, 5, gen.INT, -15, 15)
+    B_h = gen.dense(A_h.n_cols, J, 5, gen.INT, -15, 15)
     A = lf.Csr.from_host(A_h)
     M = lf.CellMatrix.build(A, lf.make_params(1, 5))
     Bd = torch.from_numpy(B_h).cuda()
     monkeypatch.setenv("LF_GROUPED", "0")
+    monkeypatch.setenv("LF_MMA", "0")
     C0 = M.spmm(Bd).cpu().numpy()
-    monkeypatch.setenv("LF_GROUPED", "1")
+    monkeypatch.setenv(env, "1")
     for _ in range(3):
         assert np.array_equal(M.spmm(Bd).cpu().numpy(), C0)
 
