@@ -220,13 +220,16 @@ LF_API lf_status lf_predict(const double features[8], int32_t max_parts, int32_t
 
 /* CSR -> CELL conversion on the GPU (section 4; canonical layout R1-R7; the
  * output is bit-identical to the oracle's).  Allocates the handle's arrays
- * through al (NULL = cudaMallocAsync).
+ * (one pool) through al (NULL = cudaMallocAsync); the temporary scratch of
+ * the conversion comes from the device's cudaMallocAsync pool on s.
  *   stats   (host, may be NULL) the statistics lf_cell_configure returned for
  *           the SAME A with params->n_parts partitions: the bucket sizes follow
  *           from them (bucket t < e_p holds H[p][t] rows, the max bucket
  *           F[p][e_p]), so the build enqueues everything asynchronously with
  *           no host synchronisation.  NULL: the sizes are counted on the GPU
- *           and s is synchronised once.
+ *           and s is synchronised once.  stats->spmm_grouped = 1 makes the
+ *           handle's lf_spmm take the grouped path (LF_GROUPED=0/1 in the
+ *           environment overrides it per call).
  * The handle may be used on s immediately.
  * Errors: LF_ERR_INVALID_ARG (sizes, e_p > k_p, P out of range, stats for a
  *         different P), LF_ERR_INDEX_OVERFLOW (n_rows >= 2^28 or K > 2^31-1),

@@ -457,7 +457,10 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
                  s_tc = up((size_t)P * lf::kMaxT * std::max(n_tiles, 1) * 8), s_kt = up((size_t)P * lf::kMaxT * 8),
                  s_rc = up((size_t)std::max<int64_t>(I, 1) * 4);
     const size_t s_head = s_seg + s_tc + s_kt + s_rc;
-    Scratch sc{mem, {}};
+    // build-time scratch comes from the device's stream-ordered pool (as the
+    // configure scratch): no allocator callback into the caller's runtime for
+    // memory that lives only until the end of this call
+    Scratch sc{Mem{nullptr, s}, {}};
     std::vector<long long> tot((size_t)P * lf::kMaxT, 0);
     if (stats) {  // bucket sizes from the configure statistics: no synchronisation
         for (int p = 0; p < P; p++) {
