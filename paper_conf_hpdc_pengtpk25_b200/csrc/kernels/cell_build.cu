@@ -219,7 +219,7 @@ __global__ void pad_init_kernel(const BucketDev *__restrict__ bk, int nb, int32_
 constexpr int kSlotThreads = 256;
 constexpr int kMaxSmemBuckets = 2048;
 #ifndef LF_SLOTS_PER_LANE
-#define LF_SLOTS_PER_LANE 4  // measured: 8 same, 16 slower (c2)
+#define LF_SLOTS_PER_LANE 8  // measured (us, c2/c3/c4): 4 -> 71/207/585, 8 -> 70/199/525, 16 slower
 #endif
 constexpr int kSlotsPerLane = LF_SLOTS_PER_LANE;    // consecutive slots per lane: 16-byte stores
 constexpr int kSlotsPerWarp = 32 * kSlotsPerLane;   // a warp's chunk
