@@ -76,12 +76,12 @@ __device__ __forceinline__ void block_len_stats(unsigned long long mn, unsigned 
 // (warp-aggregated: __match_any_sync for H, REDUX for F) and the Table 2
 // row-length statistics.
 #ifndef LF_MARK_TILE
-#define LF_MARK_TILE 4096
+#define LF_MARK_TILE 4096  // items (row ends + nonzeros) per block of the marking pass
 #endif
 constexpr int kMarkTile = LF_MARK_TILE;
 #ifndef LF_MARK_MIN_BLOCKS
-#define LF_MARK_MIN_BLOCKS 4
-#endif  // nonzeros per block of the marking pass
+#define LF_MARK_MIN_BLOCKS 4  // resident marking blocks per SM (64 registers)
+#endif
 
 __global__ void __launch_bounds__(kThreads) stats_rows_kernel(const int64_t *__restrict__ row_ptr,
                                                               const int32_t *__restrict__ col, int64_t n_rows,
