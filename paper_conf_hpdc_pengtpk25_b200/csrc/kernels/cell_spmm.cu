@@ -868,7 +868,10 @@ cudaError_t run_csr_j(const lf_csr &A, const float *B, int64_t ldb, int J, float
 // CELL row is the whole C row, red.add otherwise (kRowRun rows pre-zeroed).
 constexpr int kGR = kGroupRows;  // CELL rows per group
 constexpr int kHT = 256;   // hash slots per warp (>= kGR * 32 distinct columns)
-constexpr int kGPad = 16;  // entry lists padded to a multiple of G * U (<= 16)
+#ifndef LF_GROUP_U
+#define LF_GROUP_U 2  // distinct columns in flight per lane group (grouped path; 2 measured 1-4% faster than 4)
+#endif
+constexpr int kGPad = 4 * LF_GROUP_U;  // entry lists padded to a multiple of G * U (G <= 4)
 struct GroupStage {
     int32_t key[kHT];      // column in hash slot, -1 = free
     int32_t idx_of[kHT];   // entry index of the slot's column
@@ -888,7 +891,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, LF_GROUP_MIN_BLOCKS) cell
     using V = typename Cx::V;
     using VT = typename Cx::VT;
     using L = Layout<4, G, NV>;
-    constexpr int U = 4;  // distinct columns in flight per lane group
+    constexpr int U = LF_GROUP_U;
     static_assert(G * U <= kGPad, "entry padding");
     __shared__ __align__(16) GroupStage gs_all[kWarpsPerBlock];
     const int lane = threadIdx.x & 31;
