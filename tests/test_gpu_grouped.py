@@ -137,3 +137,19 @@ def test_grouped_heuristic(lf, monkeypatch, name, want):
     C = M.spmm(torch.from_numpy(B_h).cuda()).cpu().numpy().astype(np.float64)
     Cref, Cabs = oracle.spmm_csr(A_h, B_h)
     assert np.all(np.abs(C - Cref) <= TOL * Cabs)
+
+
+@pytest.mark.parametrize("J,ldb,ldc", [(64, 68, 72), (128, 132, 256), (32, 36, 32), (60, 64, 64)])
+def test_grouped_strided(lf, grouped, J, ldb, ldc):
+    """Row strides ldb / ldc > J (16-byte multiples: the grouped paths run;
+    J = 60 is not a multiple of 64, so the tensor-core path falls back)."""
+    A_h = gen.banded(3000, 12, seed=7, kind=gen.INT, lo=-3, hi=3)
+    B_h = gen.dense(A_h.n_cols, J, 7, gen.INT, -15, 15)
+    A = lf.Csr.from_host(A_h)
+    M = lf.CellMatrix.build(A, lf.make_params(1, 5))
+    big = torch.full((A_h.n_cols, ldb), float("nan"), device="cuda")
+    big[:, :J] = torch.from_numpy(B_h).cuda()
+    out = torch.full((A_h.n_rows, ldc), float("nan"), device="cuda")[:, :J]
+    C = M.spmm(big[:, :J], out=out).cpu().numpy().astype(np.float64)
+    Cref, _ = oracle.spmm_csr(A_h, B_h)
+    assert np.array_equal(C, Cref)
