@@ -359,10 +359,13 @@ __device__ __forceinline__ void cp_wait1() { asm volatile("cp.async.wait_group 1
 // claim is issued one range ahead and read (shuffle from lane 0) only when
 // the warp moves on, so the atomic's latency is hidden; claims grow per warp,
 // so bucket cursors only move forward.
-__device__ __forceinline__ int claim_size(int64_t n, int64_t hint, int64_t nw) {
+__device__ __forceinline__ int claim_size(int64_t n, int64_t hint, int64_t nw, int chunk = kChunk) {
     const int64_t left = n - hint;
-    return (int)max((int64_t)1, min((int64_t)kChunk, left / (2 * nw)));
+    return (int)max((int64_t)1, min((int64_t)chunk, left / (2 * nw)));
 }
+#ifndef LF_GROUP_CHUNK
+#define LF_GROUP_CHUNK 8  // groups per claim on the grouped path
+#endif
 __device__ __forceinline__ unsigned long long claim_issue(unsigned long long *ctr, int size, int lane) {
     return lane == 0 ? atomicAdd(ctr, (unsigned long long)size) : 0ull;
 }
@@ -907,7 +910,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, LF_GROUP_MIN_BLOCKS) cell
     const unsigned lt = (1u << lane) - 1u;
     const int64_t n = a.n_groups;
     int bcur = 0;
-    int sz = claim_size(n, 0, nw);
+    int sz = claim_size(n, 0, nw, LF_GROUP_CHUNK);
     int64_t g = claim_get(claim_issue(a.ctr + 1, sz, lane));
     int64_t gend = min(g + sz, n);
     while (g < n) {
@@ -997,7 +1000,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, LF_GROUP_MIN_BLOCKS) cell
         }
         __syncwarp();
         if (++g >= gend) {
-            sz = claim_size(n, g, nw);
+            sz = claim_size(n, g, nw, LF_GROUP_CHUNK);
             g = claim_get(claim_issue(a.ctr + 1, sz, lane));
             gend = min(g + sz, n);
         }
