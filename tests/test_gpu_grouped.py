@@ -153,3 +153,27 @@ def test_grouped_strided(lf, grouped, J, ldb, ldc):
     C = M.spmm(big[:, :J], out=out).cpu().numpy().astype(np.float64)
     Cref, _ = oracle.spmm_csr(A_h, B_h)
     assert np.array_equal(C, Cref)
+
+
+def test_grouped_edge_cases(lf, grouped):
+    """No entries (C exactly +0.0), fewer rows than a group, one column,
+    NaN in B rows that no nonzero references (must not leak through the
+    zero-valued entries of a group)."""
+    A_h = gen.CSR(7, 5, np.zeros(8, np.int64), np.zeros(0, np.int32), np.zeros(0, np.float32))
+    M = lf.CellMatrix.build(lf.Csr.from_host(A_h), lf.make_params(1, 2))
+    C = M.spmm(torch.full((5, 64), 3.0, device="cuda"), out=torch.full((7, 64), float("nan"), device="cuda"))
+    assert torch.equal(C, torch.zeros(7, 64, device="cuda"))
+    for I, K in ((1, 1), (3, 1), (3, 40), (5, 2)):
+        A_h = gen.random_small(I, K, 30, I + K, dup=True, zeros=True, kind=gen.INT)
+        B_h = gen.dense(K, 64, 3, gen.INT, -15, 15)
+        C, _ = run(lf, A_h, B_h, 1, 5)
+        Cref, _ = oracle.spmm_csr(A_h, B_h)
+        assert np.array_equal(C, Cref)
+    # rows 0..3 use columns {0, 1} / {2} only: B rows 3.. hold NaN and are never read
+    A_h = gen.CSR(4, 6, np.array([0, 2, 3, 4, 5], np.int64), np.array([0, 1, 2, 0, 1], np.int32),
+                  np.array([1, 2, 3, 4, 5], np.float32))
+    B_h = np.full((6, 64), np.nan, np.float32)
+    B_h[:3] = gen.dense(3, 64, 4, gen.INT, -15, 15)
+    C, _ = run(lf, A_h, B_h, 1, 5)
+    Cref, _ = oracle.spmm_csr(A_h, np.nan_to_num(B_h))
+    assert np.array_equal(C, Cref)
