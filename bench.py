@@ -398,7 +398,10 @@ def main():
         "phases_ms": ph,
         "spmm_only": {"ms": spmm_ms, "gflops": flops / (spmm_ms * 1e-3) / 1e9,
                       "hbm_gbs_alg": bytes_alg / (spmm_ms * 1e-3) / 1e9},
-        "roofline": {"kernel": "lf_spmm (zero_rows + cell_spmm_kernel)", "bound": "hbm",
+        "roofline": {"kernel": "lf_spmm (zero_rows + " + ("csr_spmm_kernel" if not params.use_cell else
+                                                          "cell_spmm_grouped_kernel" if stats.spmm_grouped and
+                                                          os.environ.get("LF_GROUPED", "") != "0" else
+                                                          "cell_spmm_kernel") + ")", "bound": "hbm",
                      "achieved": bytes_alg / world / (sp_ms * 1e-3) / 1e9, "peak": hbm_peak, "unit": "GB/s",
                      "frac": bytes_alg / world / (sp_ms * 1e-3) / 1e9 / hbm_peak, "peak_kind": peak_kind,
                      "bytes_alg_per_launch": bytes_alg // world,
