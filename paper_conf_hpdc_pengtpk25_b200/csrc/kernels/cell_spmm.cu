@@ -12,8 +12,9 @@
 //   * the lanes split J: J/4 float4 columns over 32/G lanes, G lane groups
 //     each taking every G-th slot (G = 4, 2, 1 for J <= 32, 64, >= 128); NV
 //     float4 per lane cover J up to 512 per pass (J tiles beyond that);
-//   * slot (col, val) pairs are broadcast with shuffles; B rows are gathered
-//     as float4 through the read-only path, U slots in flight per lane;
+//   * each 32-slot chunk is staged by cp.async and resolved once into B-row
+//     addresses + values in shared memory (broadcast reads); B rows are
+//     gathered as float4 through the read-only path, U slots in flight per lane;
 //   * the index/value/tag streams and C stores carry an L2 evict_first policy
 //     so the L2 keeps B rows;
 //   * the row width W is a template parameter for W <= 32, so the fold /
@@ -24,6 +25,9 @@
 //     otherwise (run split between warps, or P > 1) red.global.add.v4.f32 into
 //     the row zeroed beforehand by zero_rows_kernel (reading R11);
 //   * rows of A with no CELL row are zeroed by zero_rows_kernel (R13).
+// Alternative executions of the same CELL arrays (chosen per handle, below):
+// the grouped path (4 CELL rows per warp, one gather per distinct column) and
+// its tensor-core variant (opt-in); C is the same up to fp32 summation order.
 // Row tag (built by bucket_kernel<1>): (i << 3) | S<<2 | F<<1 | L, where F/L
 // mark the first/last sub-row of the (row, partition) segment and S that the
 // segment holds all of the row's CELL rows; -1 = padding row.

@@ -6,11 +6,17 @@
 //   Unat[p][t], Utop[p][t]   the |set(Ind)| terms of eq. 7
 // plus the Table 2 row-length statistics.  Three passes:
 //   stats_rows_kernel   one thread per row: segments, H, F (warp-aggregated),
-//                       features; t0 of every segment -> t0seg
-//   stats_mark_kernel   nnz-balanced: every nonzero sets bit t0 of its segment
-//                       in the per-column mask M[c] (partition of c is c / S)
-//   stats_cols_kernel   one thread per column: Unat[p][t] = #{c : bit t},
-//                       Utop[p][t] = #{c : highest bit >= t} (warp-aggregated)
+//                       features; t0 of every segment -> t0seg; merge-path
+//                       tiles of the marking pass
+//   stats_mark_kernel   nnz-balanced tiles: every nonzero sets bit t0 of its
+//                       segment in the per-column mask M[c] (partition of c
+//                       is c / S); tiles of one natural bucket merge their
+//                       (column, bits) pairs in a shared-memory filter first
+//   stats_cols_kernel   one thread per mask slot: Unat[p][t] = #{c : bit t},
+//                       Utop[p][t] = #{c : highest bit >= t} (bit transpose)
+// and, for the grouped SpMM path's decision, group_sample_kernel (sampled
+// distinct columns of 4-row groups); features_kernel reads the row lengths
+// alone when the statistics pass is not run speculatively (lf_api.cu).
 #include "../lf_internal.cuh"
 
 namespace lf {
