@@ -83,7 +83,31 @@ template <int VEC> struct Vec;
 template <> struct Vec<4> {
     using T = float4;
     static __device__ __forceinline__ T zero() { return make_float4(0.f, 0.f, 0.f, 0.f); }
-    static __device__ __forceinline__ T load(const float *p) { return __ldg(reinterpret_cast<const float4 *>(p)); }
+#ifndef LF_BLOAD
+#define LF_BLOAD 0  // B-row gathers: 0 = ld.global.nc; 1 = + L1::no_allocate; 2 = + L2 evict_last; 3 = L1 alloc + evict_last
+#endif
+    static __device__ __forceinline__ T load(const float *p) {
+#if LF_BLOAD == 0
+        return __ldg(reinterpret_cast<const float4 *>(p));
+#else
+        T v;
+#if LF_BLOAD == 1
+        asm("ld.global.nc.L1::no_allocate.v4.f32 {%0, %1, %2, %3}, [%4];"
+            : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p));
+#else
+        uint64_t pl;
+        asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pl));
+#if LF_BLOAD == 2
+        asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%4], %5;"
+            : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p), "l"(pl));
+#else
+        asm("ld.global.nc.L2::cache_hint.v4.f32 {%0, %1, %2, %3}, [%4], %5;"
+            : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w) : "l"(p), "l"(pl));
+#endif
+#endif
+        return v;
+#endif
+    }
     static __device__ __forceinline__ void fma(T &acc, float a, const T &b) {
         acc.x = fmaf(a, b.x, acc.x);
         acc.y = fmaf(a, b.y, acc.y);

@@ -171,7 +171,16 @@ __global__ void __launch_bounds__(kThreads) stats_rows_kernel(const int64_t *__r
 #define LF_MARK_MODE 3  // tiles of one natural bucket: 3 = block smem filter, then one RED per column;
                         // other tiles: 0 = L2 check then RED, 2 = L1-cached check, 1 / 3 = RED only
 #endif
-constexpr int kMarkFilter = 2048;            // direct-mapped (column, bits) slots per block (mode 3)
+#ifndef LF_MARK_FILTER
+#define LF_MARK_FILTER 2048
+#endif
+#ifndef LF_MARK_FBITS16
+#define LF_MARK_FBITS16 0  // 1: filter bits packed two 16-bit halves per word (twice the slots in 48 KB)
+#endif
+#ifndef LF_MARK_FILTER_ALL
+#define LF_MARK_FILTER_ALL 0  // 1: R-MAT-type tiles (several natural buckets) also go through the filter
+#endif
+constexpr int kMarkFilter = LF_MARK_FILTER;  // direct-mapped (column, bits) slots per block (mode 3)
 constexpr uint32_t kFilterEmpty = 0xFFFFFFFFu;
 constexpr uint32_t kHashOdd = LF_MARK_HASH ? 0x9E3779B1u : 1u;
 __device__ __forceinline__ uint32_t hslot(int32_t c, uint32_t kmask) { return ((uint32_t)c * kHashOdd) & kmask; }
@@ -191,10 +200,11 @@ __global__ void __launch_bounds__(kThreads, LF_MARK_MIN_BLOCKS) stats_mark_kerne
     __shared__ int32_t cnt[kMarkTile];     // rows starting at a tile position -> inclusive scan
     __shared__ uint8_t rt0[kMarkTile + 1]; // t0 of the tile's rows (P == 1)
     __shared__ int32_t wsum[kThreads / 32];
-    __shared__ uint32_t fkey[kMarkFilter], fbits[kMarkFilter];  // block filter of uniform tiles
+    constexpr int kFB = LF_MARK_FBITS16 ? kMarkFilter / 2 : kMarkFilter;
+    __shared__ uint32_t fkey[kMarkFilter], fbits[kFB];  // block filter of uniform tiles
     for (int q = threadIdx.x; q < kMarkFilter; q += blockDim.x) {
         fkey[q] = kFilterEmpty;
-        fbits[q] = 0u;
+        if (q < kFB) fbits[q] = 0u;
     }
     constexpr int K = kMarkTile / kThreads;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
@@ -292,7 +302,7 @@ __global__ void __launch_bounds__(kThreads, LF_MARK_MIN_BLOCKS) stats_mark_kerne
     uint32_t h[K];
 #pragma unroll
     for (int k = 0; k < K; k++) h[k] = c[k] >= 0 ? hslot(c[k], kmask) : 0u;
-    if (LF_MARK_MODE == 3 && uni) {
+    if (LF_MARK_MODE == 3 && (uni || LF_MARK_FILTER_ALL)) {
         // block-level merge (tiles of one natural bucket: banded / stencil
         // rows, where a tile of ~4096 nonzeros covers ~200 distinct columns):
         // (column, bits) pairs collect in a direct-mapped shared-memory filter
@@ -308,8 +318,10 @@ __global__ void __launch_bounds__(kThreads, LF_MARK_MIN_BLOCKS) stats_mark_kerne
                 cur = atomicCAS(&fkey[f], kFilterEmpty, (uint32_t)c[k]);
                 if (cur == kFilterEmpty) cur = (uint32_t)c[k];
             }
-            if (cur == (uint32_t)c[k]) {
-                if ((reinterpret_cast<volatile uint32_t *>(fbits)[f] & bit[k]) != bit[k]) atomicOr(&fbits[f], bit[k]);
+            if (cur == (uint32_t)c[k] && (!LF_MARK_FBITS16 || bit[k] < 0x10000u)) {
+                const int fw = LF_MARK_FBITS16 ? f >> 1 : f;
+                const uint32_t fb = LF_MARK_FBITS16 ? bit[k] << ((f & 1) * 16) : bit[k];
+                if ((reinterpret_cast<volatile uint32_t *>(fbits)[fw] & fb) != fb) atomicOr(&fbits[fw], fb);
             } else {
                 atomicOr(mask + h[k], bit[k]);  // slot taken by another column
             }
@@ -317,7 +329,8 @@ __global__ void __launch_bounds__(kThreads, LF_MARK_MIN_BLOCKS) stats_mark_kerne
         __syncthreads();
         for (int f = threadIdx.x; f < kMarkFilter; f += blockDim.x) {
             const uint32_t key = fkey[f];
-            if (key != kFilterEmpty) atomicOr(mask + hslot((int32_t)key, kmask), fbits[f]);
+            const uint32_t fb = LF_MARK_FBITS16 ? (fbits[f >> 1] >> ((f & 1) * 16)) & 0xFFFFu : fbits[f];
+            if (key != kFilterEmpty && fb) atomicOr(mask + hslot((int32_t)key, kmask), fb);
         }
         return;
     }
