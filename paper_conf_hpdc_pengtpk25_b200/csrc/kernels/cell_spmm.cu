@@ -784,9 +784,13 @@ __global__ void zero_rows_kernel(const uint8_t *__restrict__ row_mode, int64_t n
                    policy_evict_first());
 }
 
+#ifndef LF_CARVEOUT
+#define LF_CARVEOUT -1  // >= 0: preferred shared-memory carveout (percent of the unified L1/smem) of the SpMM kernels
+#endif
 template <typename F>
 int resident_blocks(F fn) {
     int occ = 0, sms = 0, dev = 0;
+    if (LF_CARVEOUT >= 0) cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, LF_CARVEOUT);
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kWarpsPerBlock * 32, 0);
