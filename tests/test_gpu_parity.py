@@ -338,3 +338,32 @@ def test_host_pipeline_overlapped(lf):
     for i, hC in outs:
         A_h, B_h = probs[i]
         assert np.array_equal(hC.numpy().astype(np.float64), oracle.spmm_csr(A_h, B_h)[0])
+
+
+@pytest.mark.parametrize("n_lanes", [2, 3])
+def test_steps_in_flight_on_lanes(lf, n_lanes):
+    """bench.py's pipelined steps: configure -> build -> SpMM of the SAME A issued
+    on alternating streams, each lane with its own C, the previous step's SpMM
+    still running when the next step's configure and build synchronise the
+    host; every step's result is exact."""
+    A_h = gen.rmat(13, 16, seed=11, kind=gen.INT)
+    J = 64
+    B_h = gen.dense(A_h.n_cols, J, 11, gen.INT)
+    A = lf.Csr.from_host(A_h)
+    B = torch.from_numpy(B_h).cuda()
+    ref = oracle.spmm_csr(A_h, B_h)[0]
+    lanes = [torch.cuda.current_stream()] + [torch.cuda.Stream() for _ in range(n_lanes - 1)]
+    torch.cuda.synchronize()
+    got = []
+    for it in range(4 * n_lanes):
+        st = lanes[it % n_lanes]
+        with torch.cuda.stream(st):
+            C = torch.full((A_h.n_rows, J), float("nan"), device="cuda")
+            params, stats = lf.configure(A, J, stream=st)
+            M = lf.CellMatrix.build(A, params, stats, stream=st)
+            M.spmm(B, out=C, stream=st)
+            M.close()
+        got.append(C)
+    torch.cuda.synchronize()
+    for C in got:
+        assert np.array_equal(C.cpu().numpy().astype(np.float64), ref)
