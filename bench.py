@@ -50,8 +50,8 @@ GATHER_CEILING = {"c2_rmat20": (20649.0, "profiles/r1_gather_replay.md: c2 colum
 
 # DRAM bytes per lf_spmm launch (dram__bytes_read.sum + dram__bytes_write.sum
 # of cell_spmm_kernel, ncu --set full, profiles/r1_bench_summary.md)
-NCU_TRAFFIC = {"c2_rmat20": (1496965000 + 535886848, "ncu --set full of cell_spmm_kernel (round 1, r1g): "
-                                                      "1.497 GB read + 0.536 GB written"),
+NCU_TRAFFIC = {"c2_rmat20": (1500573000 + 535747072, "ncu --set full of cell_spmm_kernel (round 1, r1m): "
+                                                      "1.501 GB read + 0.536 GB written"),
                "c3_stencil126": (1060587000 + 483531008, "ncu --set full of cell_spmm_grouped_kernel (round 1, "
                                                           "grp2_stencil64): 1.061 GB read + 0.484 GB written")}
 
