@@ -794,6 +794,11 @@ int resident_blocks(F fn) {
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kWarpsPerBlock * 32, 0);
+#ifndef LF_SPMM_GRID_BPS
+#define LF_SPMM_GRID_BPS 0  // > 0: SpMM grids hold at most this many blocks per SM (the rest of the SM is left to
+                            // kernels of other streams, e.g. the next step's configure / build)
+#endif
+    if (LF_SPMM_GRID_BPS > 0) occ = std::min(occ, LF_SPMM_GRID_BPS);
     return std::max(1, occ) * std::max(1, sms);
 }
 
