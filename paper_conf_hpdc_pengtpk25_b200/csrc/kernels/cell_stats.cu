@@ -540,7 +540,10 @@ cudaError_t launch_stats(const lf_csr &A, int P, StatsDev *d_stats, uint32_t *d_
     const size_t hist = 2 * (size_t)P * kMaxT * sizeof(unsigned long long);
     if (A.n_rows > 0) {
         const int64_t want = (A.n_rows + kThreads - 1) / kThreads;
-        const int grid = (int)std::min<int64_t>(want, (int64_t)num_sms() * 8);
+#ifndef LF_STATS_ROWS_BPS
+#define LF_STATS_ROWS_BPS 8  // stats_rows_kernel grid: at most this many blocks per SM (grid-stride over rows)
+#endif
+        const int grid = (int)std::min<int64_t>(want, (int64_t)num_sms() * LF_STATS_ROWS_BPS);
         const int64_t tiles = (A.nnz + A.n_rows + kMarkTile - 1) / kMarkTile;
         if (tiles > 0x7fffffff) return cudaErrorInvalidValue;
         int64_t *tile_row = reinterpret_cast<int64_t *>(d_t0seg + (((size_t)A.n_rows * P + 15) & ~size_t(15)));
