@@ -62,7 +62,7 @@ __device__ __forceinline__ void segment_of(const int64_t *__restrict__ row_ptr, 
 // A row folded into more than kThreadSubRows CELL rows has its sub-rows
 // written by the whole warp (coalesced) instead of by its own thread.
 #ifndef LF_THREAD_SUBROWS
-#define LF_THREAD_SUBROWS 32
+#define LF_THREAD_SUBROWS 8  // measured (bucket_kernel<0>+<1> mean, us, c2/c3/c4): 32 -> 15.2/18.6/23.0, 8 -> 14.3/18.6/22.5, 4 -> 14.4/18.3/22.0, 1 -> 15.9/17.1/28.4
 #endif
 constexpr int kThreadSubRows = LF_THREAD_SUBROWS;
 template <int PASS>
