@@ -72,6 +72,8 @@ def _L():
         _lib.lfo_build_buckets_literal.restype = _I64
         _lib.lfo_partition_stats.argtypes = [_I64, _I64, _P, _P, _I32, _I32, _P, _P, _P, _P]
         _lib.lfo_features.argtypes = [_I64, _I64, _P, _P]
+        _lib.lfo_set_threads.argtypes = [_I32]
+        _lib.lfo_set_threads.restype = _I32
     return _lib
 
 
@@ -217,3 +219,9 @@ def features(A) -> np.ndarray:
     out = np.zeros(7, np.float64)
     _L().lfo_features(A.n_rows, A.n_cols, prp, out.ctypes.data)
     return out
+
+
+def set_threads(n: int = 0) -> int:
+    """OpenMP threads of the oracle's parallel loops (n <= 0: unchanged);
+    returns the count now in effect."""
+    return int(_L().lfo_set_threads(int(n)))

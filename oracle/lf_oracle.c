@@ -25,6 +25,9 @@
 #include <stdint.h>
 #include <stdlib.h>
 #include <string.h>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
 
 /* ---------------------------------------------------------------------- */
 /* Algorithm 1, eq. 3:                            */
@@ -251,25 +254,38 @@ int64_t lfo_cell_to_csr(int64_t I, int32_t n_buckets, const lfo_bucket *buckets,
 /* ---------------------------------------------------------------------- */
 void lfo_cell_spmm(int64_t I, int64_t J, int32_t n_buckets, const lfo_bucket *buckets, const int32_t *rowInd,
                    const int32_t *colIndC, const float *valC, const float *B, int64_t ldb, double *C) {
-    for (int64_t q = 0; q < I * J; q++) C[q] = 0.0;
-    for (int32_t b = 0; b < n_buckets; b++) {
-        int64_t W = (int64_t)1 << buckets[b].width_log2;
-        int64_t R = buckets[b].rows_per_block;
-        int64_t n_blocks = buckets[b].n_rows_pad / R;
-        for (int64_t blk = 0; blk < n_blocks; blk++) {
-            for (int64_t iBlk = 0; iBlk < R; iBlk++) {
-                int64_t r = buckets[b].row_off + blk * R + iBlk;
-                int64_t i = rowInd[r];
-                if (i < 0) continue;
-                for (int64_t j = 0; j < J; j++) {
-                    double local = 0.0;
-                    for (int64_t kBlk = 0; kBlk < W; kBlk++) {
-                        int64_t s = buckets[b].slot_off + (blk * R + iBlk) * W + kBlk;
-                        int64_t kk = colIndC[s];
-                        if (kk < 0) continue;
-                        local += (double)valC[s] * (double)B[kk * ldb + j];
+    /* Threads split the j range (the output columns): every thread walks all
+     * blocks in Alg. 2's order for its own columns, so each C[i][j] receives
+     * the same additions in the same order whatever the thread count. */
+#pragma omp parallel
+    {
+        int64_t nt = 1, id = 0;
+#ifdef _OPENMP
+        nt = omp_get_num_threads();
+        id = omp_get_thread_num();
+#endif
+        const int64_t j0 = J * id / nt, j1 = J * (id + 1) / nt;
+        for (int64_t i = 0; i < I; i++)
+            for (int64_t j = j0; j < j1; j++) C[i * J + j] = 0.0;
+        for (int32_t b = 0; b < n_buckets && j0 < j1; b++) {
+            int64_t W = (int64_t)1 << buckets[b].width_log2;
+            int64_t R = buckets[b].rows_per_block;
+            int64_t n_blocks = buckets[b].n_rows_pad / R;
+            for (int64_t blk = 0; blk < n_blocks; blk++) {
+                for (int64_t iBlk = 0; iBlk < R; iBlk++) {
+                    int64_t r = buckets[b].row_off + blk * R + iBlk;
+                    int64_t i = rowInd[r];
+                    if (i < 0) continue;
+                    for (int64_t j = j0; j < j1; j++) {
+                        double local = 0.0;
+                        for (int64_t kBlk = 0; kBlk < W; kBlk++) {
+                            int64_t s = buckets[b].slot_off + (blk * R + iBlk) * W + kBlk;
+                            int64_t kk = colIndC[s];
+                            if (kk < 0) continue;
+                            local += (double)valC[s] * (double)B[kk * ldb + j];
+                        }
+                        C[i * J + j] += local;
                     }
-                    C[i * J + j] += local;
                 }
             }
         }
@@ -290,10 +306,17 @@ void lfo_cell_spmm(int64_t I, int64_t J, int32_t n_buckets, const lfo_bucket *bu
 int64_t lfo_partition_cost(int64_t I, int64_t K, const int64_t *rowPtr, const int32_t *colInd, int32_t P,
                            int32_t p, int32_t e, int64_t J) {
     if (e < 0 || e > 30) return -1;
-    int32_t *stamp = (int32_t *)calloc((size_t)(K > 0 ? K : 1), sizeof(int32_t));
-    if (!stamp) return -1;
     int64_t total = 0;
+    int failed = 0;
+    /* the buckets t = 0..e are independent sets: one thread (and one stamp
+     * array) per bucket; the int64 sum does not depend on the order */
+#pragma omp parallel for schedule(dynamic, 1) reduction(+ : total, failed)
     for (int t = 0; t <= e; t++) {
+        char *seen = (char *)calloc((size_t)(K > 0 ? K : 1), 1);
+        if (!seen) {
+            failed++;
+            continue;
+        }
         int64_t W = (int64_t)1 << t;
         int64_t I1 = 0, U = 0;
         for (int64_t i = 0; i < I; i++) {
@@ -306,17 +329,17 @@ int64_t lfo_partition_cost(int64_t I, int64_t K, const int64_t *rowPtr, const in
             if (ti != t) continue;
             I1 += (l + W - 1) / W;
             for (int64_t q = beg; q < end; q++) {
-                if (stamp[colInd[q]] != t + 1) {
-                    stamp[colInd[q]] = t + 1;
+                if (!seen[colInd[q]]) {
+                    seen[colInd[q]] = 1;
                     U++;
                 }
             }
         }
+        free(seen);
         if (I1 == 0) continue;
         total += 2 * I1 * W + U * J + I1 * J;
     }
-    free(stamp);
-    return total;
+    return failed ? -1 : total;
 }
 
 /* Largest natural bucket of partition p: ceil_log2(max segment length), or
@@ -450,4 +473,16 @@ void lfo_features(int64_t I, int64_t K, const int64_t *rowPtr, double *out) {
     out[4] = (double)mn;
     out[5] = (double)mx;
     out[6] = I > 0 ? sqrt(ss / (double)I) : 0.0;
+}
+
+/* Thread count of the OpenMP loops above (tests check thread-count
+ * independence; bench.py's cpu_baseline reports the count it used). */
+int32_t lfo_set_threads(int32_t n) {
+#ifdef _OPENMP
+    if (n > 0) omp_set_num_threads(n);
+    return omp_get_max_threads();
+#else
+    (void)n;
+    return 1;
+#endif
 }

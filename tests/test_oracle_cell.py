@@ -156,3 +156,62 @@ def test_bad_params():
     A = gen.random_small(5, 5, 3, 0)
     with pytest.raises(ValueError):
         oracle.csr_to_cell(A, 1, [3], [2])  # k < e
+
+
+def concat_real_slots(cell):
+    """Walk the CELL arrays in storage order (buckets partition-major, ascending
+    width, R7) and append every real slot of CELL row r (col >= 0) to its source
+    row rowInd[r], in slot order: (cols, val bits) per source row."""
+    rows = [[] for _ in range(cell.n_rows)]
+    for b in cell.buckets:
+        W = 1 << int(b["width_log2"])
+        for q in range(int(b["n_rows_pad"])):
+            r = int(b["row_off"]) + q
+            i = int(cell.row_ind[r])
+            s0 = int(b["slot_off"]) + q * W
+            cs = cell.col_ind[s0:s0 + W]
+            vs = cell.val[s0:s0 + W].view(np.int32)
+            if i < 0:
+                assert np.all(cs == -1) and np.all(vs == 0)  # padding row (R5)
+                continue
+            real = cs >= 0
+            n = int(real.sum())
+            assert np.all(real[:n]) and not np.any(real[n:])  # real slots form a prefix
+            rows[i].extend(zip(cs[:n].tolist(), vs[:n].tolist()))
+    return rows
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_slot_order_pin(seed):
+    """Reading R6 pinned WITHOUT the round trip's sort: the real slots of a
+    source row's CELL sub-rows, concatenated in storage order, ARE its CSR
+    entries in CSR order (values bit-identical), for every P, width and fold.
+    A swapped pair of sub-rows, a reversed slot order or a bucket out of
+    partition order (R7) fails this even when the round trip's stable sort
+    would hide it.  (Fig. 4.)"""
+    rng = np.random.default_rng(7000 + seed)
+    I, K = int(rng.integers(1, 60)), int(rng.integers(1, 90))
+    P = int(rng.integers(1, 9))
+    A = gen.random_small(I, K, 80, seed, dup=True, zeros=True)
+    e = rng.integers(0, 5, size=P)
+    k = e + rng.integers(0, 3, size=P)
+    cell = oracle.csr_to_cell(A, P, e, k)
+    got = concat_real_slots(cell)
+    for i in range(I):
+        a, b = int(A.row_ptr[i]), int(A.row_ptr[i + 1])
+        exp = list(zip(A.col_ind[a:b].tolist(), A.val[a:b].view(np.int32).tolist()))
+        assert got[i] == exp, i
+
+
+def test_slot_order_pin_catches_a_swap():
+    """The pin above is not vacuous: swapping two sub-rows of a folded row in
+    an otherwise valid CELL breaks it, while the sorted round trip still passes
+    when the swapped sub-rows hold distinct columns."""
+    A = gen.CSR(1, 16, np.array([0, 6], np.int64), np.arange(0, 12, 2, dtype=np.int32),
+                np.arange(1, 7, dtype=np.float32))
+    cell = oracle.csr_to_cell(A, 1, [1])  # W = 2: 3 sub-rows of 2
+    cell.col_ind[[0, 1, 2, 3]] = cell.col_ind[[2, 3, 0, 1]]
+    cell.val[[0, 1, 2, 3]] = cell.val[[2, 3, 0, 1]]
+    rp, ci, va = oracle.cell_to_csr(cell)
+    assert np.array_equal(ci, A.col_ind)  # the round trip is blind to the swap
+    assert concat_real_slots(cell)[0] != list(zip(A.col_ind.tolist(), A.val.view(np.int32).tolist()))

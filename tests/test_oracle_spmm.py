@@ -93,3 +93,23 @@ def test_alg2_bitwise_p1_no_folding():
     C1, _ = oracle.spmm_csr(A, B)
     C2 = oracle.cell_spmm(cell, B)
     assert np.array_equal(C1.view(np.int64), C2.view(np.int64))
+
+
+def test_cell_spmm_thread_count_independent():
+    """lfo_cell_spmm splits the output columns over threads: the fp64 result
+    is bit-identical with 1 thread and with all threads (float inputs, folded
+    rows, P > 1 so several CELL rows add into one C row)."""
+    A = gen.rmat(10, 16, seed=4)
+    B = gen.dense(A.n_cols, 37, 4)
+    cell = oracle.csr_to_cell(A, 3, [2, 3, 1])
+    n_all = oracle.set_threads(0)
+    try:
+        oracle.set_threads(1)
+        C1 = oracle.cell_spmm(cell, B)
+        oracle.set_threads(max(4, n_all))
+        C4 = oracle.cell_spmm(cell, B)
+    finally:
+        oracle.set_threads(n_all)
+    assert np.array_equal(C1.view(np.int64), C4.view(np.int64))
+    Cref, Cabs = oracle.spmm_csr(A, B)
+    assert np.all(np.abs(C1 - Cref) <= 1e-12 * Cabs)
