@@ -48,12 +48,55 @@ GATHER_CEILING = {"c2_rmat20": (20649.0, "profiles/r1_gather_replay.md: c2 colum
                                          "512-B row gathers, U=8, 4 blocks/SM, 0.399 ms")}
 
 
-# DRAM bytes per lf_spmm launch (dram__bytes_read.sum + dram__bytes_write.sum
-# of cell_spmm_kernel, ncu --set full, profiles/r1_bench_summary.md)
-NCU_TRAFFIC = {"c2_rmat20": (1500573000 + 535747072, "ncu --set full of cell_spmm_kernel (round 1, r1m): "
-                                                      "1.501 GB read + 0.536 GB written"),
-               "c3_stencil126": (1060587000 + 483531008, "ncu --set full of cell_spmm_grouped_kernel (round 1, "
-                                                          "grp2_stencil64): 1.061 GB read + 0.484 GB written")}
+def src_hash():
+    """sha1 over liblf.so's sources: a DRAM-traffic figure measured by ncu is
+    used only for the exact kernels it was measured on."""
+    import glob
+    import hashlib
+    h = hashlib.sha1()
+    pkg = os.path.join(ROOT, "paper_conf_hpdc_pengtpk25_b200", "csrc")
+    for f in sorted(glob.glob(os.path.join(pkg, "**", "*.cu*"), recursive=True) +
+                    glob.glob(os.path.join(pkg, "*.h")) + glob.glob(os.path.join(ROOT, "include", "*.h"))):
+        with open(f, "rb") as fh:
+            h.update(os.path.relpath(f, ROOT).encode() + b"\0" + fh.read())
+    return h.hexdigest()
+
+
+def ncu_traffic(config, J):
+    """dram__bytes_read.sum + dram__bytes_write.sum per launch of the SpMM
+    kernels (kernel-name matched) from profiles/traffic.json, written by
+    scripts/ncu_traffic.py with ncu on the SAME sources (hash checked);
+    None when absent or stale."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+            t = json.load(f)
+    except Exception:
+        return None, "profiles/traffic.json absent"
+    e = t.get("entries", {}).get(f"{config}:J{J}")
+    if not e:
+        return None, f"no ncu entry for {config} J={J}"
+    if t.get("src_hash") != src_hash():
+        return None, "profiles/traffic.json measured on other sources (stale)"
+    return int(e["dram_bytes"]), f"ncu {e['kernels']} ({t.get('when', '?')}): {e['dram_read']} B read + " \
+                                 f"{e['dram_write']} B written per launch"
+
+
+def fp32_peak_tflops():
+    """FP32 CUDA-core peak: SMs x 128 FMA/clk x 2 flop x max SM clock (B200:
+    148 x 128 x 2 x 1.965 GHz = 74.4 TFLOP/s)."""
+    sm_mhz = 1965.0
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            sm_mhz = float(json.load(f).get("sm_max_mhz", sm_mhz))
+    except Exception:
+        pass
+    n_sm = 148
+    try:
+        import torch
+        n_sm = torch.cuda.get_device_properties(torch.cuda.current_device()).multi_processor_count
+    except Exception:
+        pass
+    return n_sm * 128 * 2 * sm_mhz * 1e6 / 1e12
 
 
 def gather_roofline(config, nnz, J, world, spmm_ms):
@@ -140,7 +183,8 @@ def sample_rows(A_h, n_rows, seed=0):
 
 def oracle_step(sub, B_h, J):
     """The oracle of the whole path on a row sample: Algorithm 3 over eq. 7
-    (configure), CSR->CELL, Algorithm 2 SpMM -- all single-threaded C."""
+    (configure), CSR->CELL, Algorithm 2 SpMM -- plain C, OpenMP where the
+    oracle is parallel (eq. 7's buckets, Alg. 2's output columns)."""
     import oracle
     e, k = oracle.configure(sub, 1, J)
     cell = oracle.csr_to_cell(sub, 1, e, k)
@@ -161,14 +205,22 @@ def calibrate_sample(A_h, B_h, J, target_s):
     return sample_rows(A_h, n)
 
 
-def cpu_baseline(A_h, B_h, J, target_s=15.0):
-    sub = calibrate_sample(A_h, B_h, J, target_s)
-    t0 = time.perf_counter()
-    oracle_step(sub, B_h, J)
-    dt = time.perf_counter() - t0
-    return {"value": 2.0 * sub.nnz * J / dt / 1e9, "unit": "GFLOP/s", "cores": 1, "kind": "oracle",
+def cpu_baseline(A_h, B_h, J, target_s=15.0, threads=0):
+    """The oracle as it stands on the host's cores (threads = 0: all of them,
+    OMP default), on a bounded random row sample of the workload."""
+    import oracle
+    prev = oracle.set_threads(0)
+    cores = oracle.set_threads(threads) if threads > 0 else prev
+    try:
+        sub = calibrate_sample(A_h, B_h, J, target_s)
+        t0 = time.perf_counter()
+        oracle_step(sub, B_h, J)
+        dt = time.perf_counter() - t0
+    finally:
+        oracle.set_threads(prev)
+    return {"value": 2.0 * sub.nnz * J / dt / 1e9, "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
             "sample": f"{sub.n_rows} random rows ({sub.nnz} nnz) of the workload; oracle configure (Alg. 3 over "
-                      f"eq. 7) + CSR->CELL + Alg. 2 fp64 SpMM, single thread, {dt:.2f} s",
+                      f"eq. 7) + CSR->CELL + Alg. 2 fp64 SpMM, {cores} OpenMP thread(s), {dt:.2f} s",
             "host_cpus": os.cpu_count()}
 
 
@@ -176,6 +228,8 @@ def run_reference(args):
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return 0
+    import oracle
+    cores = oracle.set_threads(0)
     A_h, J = gen.config(args.config, args.seed)
     B_h = gen.dense(A_h.n_cols, J, args.seed)
     per_step = max(0.2, min(5.0, 120.0 / (args.steps + args.warmup)))
@@ -192,9 +246,10 @@ def run_reference(args):
             "scaling": "strong", "vs_baseline": None, "dtype": "f64", "data": "synthetic",
             "config": {"workload": args.config, "J": J, "n_rows": A_h.n_rows, "nnz": A_h.nnz,
                        "sample_rows": sub.n_rows, "sample_nnz": sub.nnz},
-            "cpu_baseline": {"value": v, "unit": "GFLOP/s", "cores": 1, "kind": "oracle",
+            "cpu_baseline": {"value": v, "unit": "GFLOP/s", "cores": cores, "kind": "oracle",
                              "sample": f"{sub.n_rows} random rows ({sub.nnz} nnz) per step; oracle configure + "
-                                       "CSR->CELL + Alg. 2 fp64, single thread"},
+                                       f"CSR->CELL + Alg. 2 fp64, {cores} OpenMP threads",
+                             "host_cpus": os.cpu_count()},
             "e2e": {"value": v, "unit": "GFLOP/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
     return 0
@@ -203,6 +258,37 @@ def run_reference(args):
 # --------------------------------------------------------------------------
 # GPU arm
 # --------------------------------------------------------------------------
+DEFAULT_EXTRA = "c3b_banded2M:128,c3b_banded2M:64,c3_stencil126:64,c3_stencil126:128,c4_reddit:256"
+
+
+def maybe_spawn(args):
+    """--gpus N > 1 outside torchrun: launch N ranks with torch.distributed.run
+    on this node (127.0.0.1) and return its exit code; fail loudly when the
+    node has fewer GPUs.  Inside torchrun, WORLD_SIZE must equal N."""
+    ws = os.environ.get("WORLD_SIZE")
+    if ws is not None:
+        if int(ws) != args.gpus and args.gpus != 1:
+            print(f"bench.py: --gpus {args.gpus} but WORLD_SIZE={ws}", file=sys.stderr)
+            return 2
+        return None
+    if args.gpus <= 1:
+        return None
+    import socket
+    import subprocess
+    import torch
+    n_dev = torch.cuda.device_count()
+    if n_dev < args.gpus:
+        print(f"bench.py: --gpus {args.gpus} requested but only {n_dev} CUDA device(s) visible", file=sys.stderr)
+        return 2
+    so = socket.socket()
+    so.bind(("127.0.0.1", 0))
+    port = so.getsockname()[1]
+    so.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__), *sys.argv[1:]]
+    return subprocess.call(cmd)
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -211,10 +297,13 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--config", default="c2_rmat20")
     ap.add_argument("--seed", type=int, default=0)
-    ap.add_argument("--parts", type=int, default=0, help="force P (0 = predictor stand-in)")
+    ap.add_argument("--parts", type=int, default=0, help="force P (0 = predictor)")
     ap.add_argument("--width-log2", type=int, default=-1, help="force e_p (-1 = Algorithm 3)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--extra", default=DEFAULT_EXTRA,
+                    help="further workloads timed in the same run, name:J comma-separated ('none' to skip): each "
+                         "gets its SpMM-only time, step time and roofline block")
     ap.add_argument("--shard-mode", default="nnz", choices=["nnz", "bytes"])
     ap.add_argument("--streams", type=int, default=2,
                     help="steps in flight: consecutive steps alternate over this many CUDA streams, each with its "
@@ -225,6 +314,9 @@ def main():
         args.warmup = 3
     if args.impl == "reference":
         return run_reference(args)
+    rc = maybe_spawn(args)
+    if rc is not None:
+        return rc
 
     import torch
     import torch.distributed as dist
@@ -238,6 +330,20 @@ def main():
     dev = torch.device("cuda", local)
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
+        assert dist.get_world_size() == world == args.gpus, "NCCL communicator size != --gpus"
+    ev = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
+
+    def maxr(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def barrier():
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
 
     A_h, J = gen.config(args.config, args.seed)
     B_h = gen.dense(A_h.n_cols, J, args.seed)
@@ -273,7 +379,6 @@ def main():
     if args.width_log2 >= 0:
         kw["force_width_log2"] = args.width_log2
 
-    ev = lambda: torch.cuda.Event(enable_timing=True)  # noqa: E731
     phase = {"configure": [], "build": [], "spmm": [], "gather": []}
     info = {}
 
@@ -294,6 +399,7 @@ def main():
         if record:
             phase["_ev"].append((e0, e1, e2, e3, e4))
             info["params"] = params.as_dict()
+            info["path"] = M.path()
             v = M.view()
             info["cell_slots"] = int(v["n_slots"])
             info["cell_rows"] = int(v["n_cell_rows"])
@@ -304,14 +410,10 @@ def main():
     phase["_ev"] = []
     for i in range(max(args.warmup, n_lanes)):  # every lane warmed (its allocator pool and C)
         step(A, lane=i % n_lanes)
-    torch.cuda.synchronize()
-    if world > 1:
-        dist.barrier()
+    barrier()
     with ClockSampler(local) as clk:
         t0 = ev(); t1 = ev()
-        torch.cuda.synchronize()
-        if world > 1:
-            dist.barrier()
+        barrier()
         t0.record(stream)
         for st in lanes[1:]:
             st.wait_event(t0)
@@ -323,9 +425,7 @@ def main():
         torch.cuda.synchronize()
     ms_serial = None
     if n_lanes > 1:  # phases (and the serial step time) from steps run one at a time on lane 0
-        torch.cuda.synchronize()
-        if world > 1:
-            dist.barrier()
+        barrier()
         u0 = ev(); u1 = ev()
         u0.record(stream)
         for _ in range(args.steps):
@@ -342,14 +442,6 @@ def main():
         phase["spmm"].append(e2.elapsed_time(e3))
         phase["gather"].append(e3.elapsed_time(e4))
     ph = {k: float(np.mean(v)) for k, v in phase.items() if k != "_ev"}
-
-    def maxr(x):
-        if world == 1:
-            return x
-        t = torch.tensor([x], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        return float(t.item())
-
     ms = maxr(ms)
     if ms_serial is not None:
         ms_serial = maxr(ms_serial)
@@ -360,7 +452,7 @@ def main():
     M = lf.CellMatrix.build(A, params, stats)
     for _ in range(3):
         M.spmm(d_B, out=C_loc)
-    torch.cuda.synchronize()
+    barrier()
     n_sp = max(10, args.steps)
     s0, s1 = ev(), ev()
     s0.record(stream)
@@ -369,6 +461,7 @@ def main():
     s1.record(stream)
     torch.cuda.synchronize()
     spmm_ms = maxr(s0.elapsed_time(s1) / n_sp)
+    M.close()
 
     # ---- e2e: host buffers in, result back, through the public API ---------
     e2e = None
@@ -385,6 +478,7 @@ def main():
         for i in range(2):
             pipe.submit(h_rp, h_ci, h_va, h_B, h_Cs[i % 2])
         pipe.synchronize()
+        barrier()
         x0, x1 = ev(), ev()
         n_e2e = max(3, min(args.steps, 20))
         x0.record(pipe.s_h2d)
@@ -396,6 +490,17 @@ def main():
         e2e = {"value": flops / (e2e_ms * 1e-3) / 1e9, "unit": "GFLOP/s", "ms_per_step": e2e_ms,
                "api": "HostPipeline.submit (host CSR + B in, host C out; N > 1: each rank's row block)",
                "h2d_bytes_per_step": int(h2d * world), "d2h_bytes_per_step": int(d2h * world)}
+        del pipe
+    del C_full, C_loc, lane_C, d_rp, d_ci, d_va, d_B, A
+    torch.cuda.empty_cache()
+
+    # ---- further workloads (BASELINE configs 3-4 and the J=128 band target) --
+    extras = []
+    if args.extra and args.extra != "none":
+        for item in args.extra.split(","):
+            name, jx = item.split(":")
+            extras.append(time_workload(lf, lfd, torch, dist, name, int(jx), args, world, rank, dev, ev, maxr,
+                                        barrier))
 
     if rank != 0:
         if world > 1:
@@ -408,8 +513,7 @@ def main():
     # predictor picks P > 1; larger -> features_kernel + group_sample first,
     # then the statistics pass when CELL is used.  build: bucket_kernel<0>,
     # tile_scan, pad_init, bucket_kernel<1>, slot_fill, run_bounds (+ seg_kernel
-    # for P > 1).  SpMM: zero_rows_kernel + cell_spmm (or grouped) kernel; the
-    # CSR format: csr_spmm_kernel only.
+    # for P > 1).  SpMM: zero_rows_kernel + the SpMM kernel; CSR: csr_spmm_kernel.
     spec = args.parts != 0 or A_h.nnz <= (1 << 25)
     cfg_launches = (4 + (4 if (params.n_parts != 1 and args.parts == 0 and params.use_cell) else 0)) if spec \
         else (2 + (4 if params.use_cell else 0))
@@ -418,40 +522,109 @@ def main():
     else:
         launches_per_step = cfg_launches + 1
     sp_ms = ph["spmm"]
+    traffic, traffic_src = ncu_traffic(args.config, J) if world == 1 else (None, "N > 1")
     line = {
         "metric": METRIC, "value": flops / (ms * 1e-3) / 1e9, "unit": "GFLOP/s", "n_gpus": world,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
         "config": {"workload": args.config, "J": J, "n_rows": A_h.n_rows, "n_cols": A_h.n_cols, "nnz": A_h.nnz,
-                   "distinct_cols": U, "params": info.get("params"), "cell_slots": info.get("cell_slots"),
+                   "distinct_cols": U, "params": info.get("params"), "spmm_path": info.get("path"),
+                   "cell_slots": info.get("cell_slots"),
                    "cell_rows": info.get("cell_rows"), "n_buckets": info.get("n_buckets"),
                    "parallelism": f"rows{world}", "shard_mode": args.shard_mode, "streams": n_lanes,
                    "l2": "inputs larger than L2 (B, C, CELL each >126 MB); no flush"},
         "phases_ms": ph,
         "ms_per_step_serial": ms_serial if ms_serial is not None else ms,
         "spmm_only": {"ms": spmm_ms, "gflops": flops / (spmm_ms * 1e-3) / 1e9,
-                      "hbm_gbs_alg": bytes_alg / (spmm_ms * 1e-3) / 1e9},
-        "roofline": {"kernel": "lf_spmm (zero_rows + " + ("csr_spmm_kernel" if not params.use_cell else
-                                                          "cell_spmm_grouped_kernel" if stats.spmm_grouped and
-                                                          os.environ.get("LF_GROUPED", "") != "0" else
-                                                          "cell_spmm_kernel") + ")", "bound": "hbm",
+                      "hbm_gbs_alg": bytes_alg / world / (spmm_ms * 1e-3) / 1e9},
+        "roofline": {"kernel": "lf_spmm: " + str(info.get("path")), "bound": "hbm",
                      "achieved": bytes_alg / world / (sp_ms * 1e-3) / 1e9, "peak": hbm_peak, "unit": "GB/s",
                      "frac": bytes_alg / world / (sp_ms * 1e-3) / 1e9 / hbm_peak, "peak_kind": peak_kind,
                      "bytes_alg_per_launch": bytes_alg // world,
-                     "traffic": NCU_TRAFFIC[args.config][0] if args.config in NCU_TRAFFIC and world == 1 else None,
-                     "traffic_source": NCU_TRAFFIC[args.config][1] if args.config in NCU_TRAFFIC and world == 1
-                     else None},
+                     "traffic": traffic, "traffic_source": traffic_src},
         "gather": gather_roofline(args.config, A_h.nnz, J, world, sp_ms),
+        "workloads": extras,
         "clocks": clk.summary(),
         "gpu_launches": launches_per_step * args.steps,
         "e2e": e2e,
     }
     if world == 1 and not args.no_cpu_baseline:
         line["cpu_baseline"] = cpu_baseline(A_h, B_h, J)
+        st1 = cpu_baseline(A_h, B_h, J, target_s=5.0, threads=1)
+        line["cpu_baseline"]["single_thread"] = {k: st1[k] for k in ("value", "cores", "sample")}
     print(json.dumps(line), flush=True)
     if world > 1:
         dist.destroy_process_group()
     return 0
+
+
+def time_workload(lf, lfd, torch, dist, name, J, args, world, rank, dev, ev, maxr, barrier):
+    """One further workload, row-sharded like the headline: SpMM-only time
+    (back-to-back lf_spmm, CUDA events, max over ranks), serial step time
+    (configure + build + SpMM) and the roofline of the bound SURVEY 8(d)
+    assigns it (HBM for c2/c3, FP32 ALU for c4)."""
+    A_h, _ = gen.config(name, args.seed)
+    B_h = gen.dense(A_h.n_cols, J, args.seed)
+    bytes_alg, U = algorithmic_bytes(A_h, J)
+    flops = 2.0 * A_h.nnz * J
+    bounds = lfd.shard_bounds(A_h.row_ptr, world, J, args.shard_mode)
+    lo, hi = int(bounds[rank]), int(bounds[rank + 1])
+    p0, p1 = int(A_h.row_ptr[lo]), int(A_h.row_ptr[hi])
+    A = lf.Csr(torch.from_numpy(A_h.row_ptr[lo:hi + 1] - p0).to(dev), torch.from_numpy(A_h.col_ind[p0:p1]).to(dev),
+               torch.from_numpy(A_h.val[p0:p1]).to(dev), A_h.n_cols, p1 - p0)
+    B = torch.from_numpy(B_h).to(dev)
+    C = torch.empty((hi - lo, J), dtype=torch.float32, device=dev)
+    for _ in range(3):
+        params, stats = lf.configure(A, J)
+        M = lf.CellMatrix.build(A, params, stats)
+        M.spmm(B, out=C)
+        M.close()
+    barrier()
+    n_st = max(5, min(args.steps, 10))
+    s0, s1 = ev(), ev()
+    s0.record()
+    for _ in range(n_st):
+        params, stats = lf.configure(A, J)
+        M = lf.CellMatrix.build(A, params, stats)
+        M.spmm(B, out=C)
+        M.close()
+    s1.record()
+    torch.cuda.synchronize()
+    step_ms = maxr(s0.elapsed_time(s1) / n_st)
+    params, stats = lf.configure(A, J)
+    M = lf.CellMatrix.build(A, params, stats)
+    for _ in range(3):
+        M.spmm(B, out=C)
+    barrier()
+    n_sp = max(10, min(args.steps, 30))
+    s0.record()
+    for _ in range(n_sp):
+        M.spmm(B, out=C)
+    s1.record()
+    torch.cuda.synchronize()
+    sp_ms = maxr(s0.elapsed_time(s1) / n_sp)
+    path = M.path()
+    M.close()
+    out = {"workload": name, "J": J, "n_rows": A_h.n_rows, "nnz": A_h.nnz, "distinct_cols": U,
+           "params": params.as_dict(), "spmm_path": path, "spmm_ms": sp_ms, "step_ms_serial": step_ms,
+           "gflops": flops / (sp_ms * 1e-3) / 1e9, "step_gflops": flops / (step_ms * 1e-3) / 1e9}
+    hbm_peak, peak_kind = peaks()
+    gbs = bytes_alg / world / (sp_ms * 1e-3) / 1e9
+    traffic, traffic_src = ncu_traffic(name, J) if world == 1 else (None, "N > 1")
+    if name.startswith("c4"):
+        # SURVEY 8(d): 42 flop/B -> the FP32 CUDA-core ALUs bound c4
+        pk = fp32_peak_tflops()
+        ach = flops / world / (sp_ms * 1e-3) / 1e12
+        out["roofline"] = {"bound": "alu", "achieved": ach, "peak": pk, "unit": "TFLOP/s", "frac": ach / pk,
+                           "peak_kind": "derived: SMs x 128 FP32 FMA/clk x 2 x max SM clock",
+                           "hbm_frac": gbs / hbm_peak, "traffic": traffic, "traffic_source": traffic_src}
+    else:
+        out["roofline"] = {"bound": "hbm", "achieved": gbs, "peak": hbm_peak, "unit": "GB/s", "frac": gbs / hbm_peak,
+                           "peak_kind": peak_kind, "bytes_alg_per_launch": bytes_alg // world, "traffic": traffic,
+                           "traffic_source": traffic_src}
+    del A, B, C
+    torch.cuda.empty_cache()
+    return out
 
 
 if __name__ == "__main__":

@@ -81,7 +81,9 @@ typedef struct lf_csr {
 /* Device-memory provider for the handle's arrays (e.g. PyTorch's caching
  * allocator).  alloc must return a 256-byte-aligned device pointer usable on
  * stream s, or NULL; free releases it (stream-ordered on s).  Passing a NULL
- * lf_allocator* uses cudaMallocAsync / cudaFreeAsync on the call's stream. */
+ * lf_allocator* uses cudaMallocFromPoolAsync / cudaFreeAsync on the call's
+ * stream with the library's private per-device memory pool (release
+ * threshold 512 MiB; the device's default pool is left untouched). */
 typedef struct lf_allocator {
     void *ctx;
     void *(*alloc)(void *ctx, size_t bytes, lf_stream_t s);
@@ -220,8 +222,8 @@ LF_API lf_status lf_predict(const double features[8], int32_t max_parts, int32_t
 
 /* CSR -> CELL conversion on the GPU (section 4; canonical layout R1-R7; the
  * output is bit-identical to the oracle's).  Allocates the handle's arrays
- * (one pool) through al (NULL = cudaMallocAsync); the temporary scratch of
- * the conversion comes from the device's cudaMallocAsync pool on s.
+ * (one pool) through al (NULL = the private pool below); the temporary scratch of
+ * the conversion comes from the library's private stream-ordered pool on s.
  *   stats   (host, may be NULL) the statistics lf_cell_configure returned for
  *           the SAME A with params->n_parts partitions: the bucket sizes follow
  *           from them (bucket t < e_p holds H[p][t] rows, the max bucket
@@ -231,8 +233,11 @@ LF_API lf_status lf_predict(const double features[8], int32_t max_parts, int32_t
  *           handle's lf_spmm take the grouped path (LF_GROUPED=0/1 in the
  *           environment overrides it per call).
  * The handle may be used on s immediately.
- * Errors: LF_ERR_INVALID_ARG (sizes, e_p > k_p, P out of range, stats for a
- *         different P), LF_ERR_INDEX_OVERFLOW (n_rows >= 2^28 or K > 2^31-1),
+ * Errors: LF_ERR_INVALID_ARG (sizes, e_p > k_p, P out of range; stats for a
+ *         different P, for a matrix with other n_rows / n_cols / nnz, or with
+ *         tables that do not cover A: sum_p F[p][0] != nnz, e.g. the stats of
+ *         a configure that chose the CSR format; with LF_VALIDATE=1 also bucket
+ *         sizes counted on the GPU that differ from the stats), LF_ERR_INDEX_OVERFLOW (n_rows >= 2^28 or K > 2^31-1),
  *         LF_ERR_NO_MEMORY, LF_ERR_CUDA, LF_ERR_UNSORTED_CSR (LF_VALIDATE=1). */
 LF_API lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_configure_stats *stats,
                                const lf_allocator *al, lf_stream_t s, lf_cell **out);
@@ -242,10 +247,19 @@ LF_API lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, co
  *   B (device) K x J, ldb >= J;   C (device) I x J, ldc >= J;   J >= 0.
  * The vectorised path needs J % 4 == 0 and 16-byte aligned B, C, ldb*4,
  * ldc*4; other shapes take the scalar path.  Asynchronous on s; no host
- * synchronisation.  The handle is immutable: concurrent calls on different
- * streams with different C are safe.  B must not alias C. */
+ * synchronisation.  The handle's arrays are immutable: concurrent calls on
+ * different streams (and host threads) with different C are safe -- the
+ * work-queue counter slot a launch uses is fenced behind that slot's previous
+ * launch when it ran on another stream.  B must not alias C. */
 LF_API lf_status lf_spmm(const lf_cell *h, const float *B, int64_t ldb, int32_t J, float *C, int64_t ldc,
                   lf_stream_t s);
+
+/* Name of the SpMM kernel family lf_spmm runs for this handle at this J
+ * with 16-byte aligned B / C and ldb = ldc = J (e.g. "cell_spmm_kernel",
+ * "cell_spmm_grouped_kernel", "cell_spmm_tc_kernel", "csr_spmm_kernel";
+ * "" for a NULL handle, J <= 0 or an empty matrix).  Host only; the string is
+ * static.  For reports and tests: it launches nothing. */
+LF_API const char *lf_spmm_kernel_name(const lf_cell *h, int32_t J);
 
 /* Algorithm 1 on the GPU directly from CSR: the fixed-format
  * path the predictor can choose instead of CELL.  Same conventions as lf_spmm. */
@@ -255,7 +269,11 @@ LF_API lf_status lf_csr_spmm(const lf_csr *A, const float *B, int64_t ldb, int32
 /* Fills *out with the handle's arrays (no copy; valid until destroy). */
 LF_API lf_status lf_cell_view(const lf_cell *h, lf_cell_arrays *out);
 
-/* Frees the handle and its arrays (stream-ordered on the build stream). */
+/* Frees the handle and its arrays, stream-ordered on the build stream after
+ * every lf_spmm of the handle on any stream (each other stream's last launch
+ * is recorded by lf_spmm and waited for here); returns without blocking.
+ * The build stream must still exist.  Not thread-safe against concurrent
+ * lf_spmm calls on the same handle. */
 LF_API lf_status lf_cell_destroy(lf_cell *h);
 
 LF_API const char *lf_status_string(lf_status st);

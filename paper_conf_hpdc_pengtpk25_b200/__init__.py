@@ -147,9 +147,15 @@ class CellMatrix:
             out = torch.empty((self.n_rows, J), dtype=torch.float32, device=B.device)
         if out.shape != (self.n_rows, J) or out.stride(1) != 1 or out.dtype != torch.float32:
             raise ValueError("out must be [I, J] float32 with unit column stride")
+        self._J = J
         _abi.check(lib.lf_spmm(self._h, B.data_ptr(), max(B.stride(0), J), J, out.data_ptr(),
                                max(out.stride(0), J), _stream(stream)))
         return out
+
+    def path(self, J: int | None = None) -> str:
+        """Kernel family lf_spmm runs for this handle (aligned B / C, ldb = ldc = J)."""
+        J = int(J if J is not None else getattr(self, "_J", 0) or 0)
+        return (lib.lf_spmm_kernel_name(self._h, J) or b"").decode()
 
     def view(self) -> dict:
         """The CELL arrays (zero-copy CUDA tensors valid while self lives) and the

@@ -85,6 +85,7 @@ SIGNATURES = {
                              ctypes.POINTER(LfAllocator), _P, ctypes.POINTER(ctypes.c_void_p)]),
     "lf_spmm": (_I32, [_P, _P, _I64, _I32, _P, _I64, _P]),
     "lf_predict": (_I32, [ctypes.POINTER(ctypes.c_double), _I32, ctypes.POINTER(_I32), ctypes.POINTER(_I32)]),
+    "lf_spmm_kernel_name": (ctypes.c_char_p, [_P, _I32]),
     "lf_csr_spmm": (_I32, [ctypes.POINTER(LfCsr), _P, _I64, _I32, _P, _I64, _P]),
     "lf_cell_view": (_I32, [_P, ctypes.POINTER(LfCellArrays)]),
     "lf_cell_destroy": (_I32, [_P]),

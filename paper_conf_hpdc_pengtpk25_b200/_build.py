@@ -30,14 +30,30 @@ def _newest(paths):
     return max((os.path.getmtime(p) for p in paths), default=0.0)
 
 
+def src_hash(defs=()) -> str:
+    """sha1 of every source and header, the flags and the -D macros: liblf.so
+    is reused only when it was built from exactly these (a stamp file next to
+    it), never on timestamps alone (a pushed or copied binary keeps its mtime)."""
+    import hashlib
+    h = hashlib.sha1(" ".join([NVCC, *ARCH, *FLAGS, *defs]).encode())
+    for f in sorted(sources() + _headers() + [__file__]):
+        with open(f, "rb") as fh:
+            h.update(os.path.relpath(f, ROOT).encode() + b"\0" + fh.read())
+    return h.hexdigest()
+
+
 def build(force: bool = False, verbose: bool = False, defs=(), out: str | None = None) -> str:
     """defs: extra -D macros (experiment variants go to `out` / build_<tag>/)."""
     global OBJ
     lib = out or LIB
     obj_dir = OBJ if not defs else OBJ + "_" + "_".join(d.replace("=", "") for d in defs)
     srcs = sources()
-    if not force and os.path.exists(lib) and os.path.getmtime(lib) >= _newest(srcs + _headers() + [__file__]):
-        return lib
+    stamp = lib + ".srchash"
+    want = src_hash(defs)
+    if not force and os.path.exists(lib) and os.path.exists(stamp):
+        with open(stamp) as f:
+            if f.read().strip() == want:
+                return lib
     os.makedirs(obj_dir, exist_ok=True)
     hdr_t = _newest(_headers() + [__file__])
 
@@ -57,6 +73,8 @@ def build(force: bool = False, verbose: bool = False, defs=(), out: str | None =
     tmp = lib + f".tmp{os.getpid()}"
     subprocess.check_call([NVCC, *ARCH, "-shared", "-o", tmp, *objs, "-cudart", "static"])
     os.replace(tmp, lib)
+    with open(stamp, "w") as f:
+        f.write(want + "\n")
     return lib
 
 

@@ -366,7 +366,7 @@ __global__ void validate_kernel(const int64_t *__restrict__ row_ptr, const int32
 
 int grid_for(int64_t n, int threads) {
     int64_t g = (n + threads - 1) / threads;
-    return (int)std::max<int64_t>(1, std::min<int64_t>(g, 148LL * 32));
+    return (int)std::max<int64_t>(1, std::min<int64_t>(g, (int64_t)sm_count() * 32));
 }
 
 }  // namespace

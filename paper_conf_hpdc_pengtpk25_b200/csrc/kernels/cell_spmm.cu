@@ -789,10 +789,9 @@ __global__ void zero_rows_kernel(const uint8_t *__restrict__ row_mode, int64_t n
 #endif
 template <typename F>
 int resident_blocks(F fn) {
-    int occ = 0, sms = 0, dev = 0;
+    int occ = 0;
+    const int sms = sm_count();
     if (LF_CARVEOUT >= 0) cudaFuncSetAttribute(fn, cudaFuncAttributePreferredSharedMemoryCarveout, LF_CARVEOUT);
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kWarpsPerBlock * 32, 0);
 #ifndef LF_SPMM_GRID_BPS
 #define LF_SPMM_GRID_BPS 0  // > 0: SpMM grids hold at most this many blocks per SM (the rest of the SM is left to
@@ -804,8 +803,9 @@ int resident_blocks(F fn) {
 
 template <int VEC, int G, int NV, bool FULL>
 cudaError_t run_cell(const SpmmArgs &a0, cudaStream_t s) {
-    static int cap = 0;
+    static int caps[64];
     auto fn = cell_spmm_kernel<VEC, G, NV, FULL>;
+    int &cap = caps[current_device()];
     if (!cap) cap = resident_blocks(fn);
     SpmmArgs a = a0;
     const int64_t per_block = kWarpsPerBlock * kChunk;
@@ -878,8 +878,9 @@ cudaError_t run_cell_j(const SpmmArgs &a, cudaStream_t s) {
 
 template <int VEC, int G, int NV, bool FULL>
 cudaError_t run_csr(const lf_csr &A, const float *B, int64_t ldb, int J, float *C, int64_t ldc, cudaStream_t s) {
-    static int cap = 0;
+    static int caps[64];
     auto fn = csr_spmm_kernel<VEC, G, NV, FULL>;
+    int &cap = caps[current_device()];
     if (!cap) cap = resident_blocks(fn);
     int64_t want = (A.n_rows + kWarpsPerBlock - 1) / kWarpsPerBlock;
     int grid = (int)std::max<int64_t>(1, std::min<int64_t>(want, cap));
@@ -1055,8 +1056,9 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, LF_GROUP_MIN_BLOCKS) cell
 
 template <int G, int NV, bool FULL>
 cudaError_t run_grouped(const SpmmArgs &a, cudaStream_t s) {
-    static int cap = 0;
+    static int caps[64];
     auto fn = cell_spmm_grouped_kernel<G, NV, FULL>;
+    int &cap = caps[current_device()];
     if (!cap) cap = resident_blocks(fn);
     const int64_t want = std::max<int64_t>((a.n_groups + kWarpsPerBlock - 1) / kWarpsPerBlock,
                                            (a.n_rows + 32 * kWarpsPerBlock - 1) / (32 * kWarpsPerBlock));
@@ -1103,7 +1105,7 @@ struct MmaStage {
     int32_t key[kMHT];
     int32_t idx_of[kMHT];
     int32_t hslot[kKCap + 32];
-    const float *caddr[kKCap + 8];
+    const float *caddr[kKCap + 32];  // entries up to kKCap + 31 are written before `over` is seen
     float V[kMR * kVStride];
 };
 
@@ -1311,14 +1313,13 @@ __global__ void __launch_bounds__(kMmaWarps * 32) cell_spmm_mma_kernel(const Spm
 
 template <int NT>
 cudaError_t run_mma(const SpmmArgs &a, cudaStream_t s) {
-    static int cap = 0;
+    static int caps[64];
     auto fn = cell_spmm_mma_kernel<NT>;
+    int &cap = caps[current_device()];
     if (!cap) {
-        int occ = 0, sms = 0, dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+        int occ = 0;
         cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, fn, kMmaWarps * 32, 0);
-        cap = std::max(1, occ) * std::max(1, sms);
+        cap = std::max(1, occ) * sm_count();
     }
     const int64_t want = std::max<int64_t>((a.n_groups_m + kMmaWarps - 1) / kMmaWarps,
                                            (a.n_rows + 32 * kMmaWarps - 1) / (32 * kMmaWarps));
@@ -1348,7 +1349,7 @@ cudaError_t zero_red_rows(const SpmmArgs &a, bool tiled, cudaStream_t s) {
     const int vec4 = (a.J % 4 == 0 && a.ldc % 4 == 0 && ((uintptr_t)a.C & 15) == 0) ? 1 : 0;
     const unsigned mask = (1u << kRowRed) | (tiled ? (1u << kRowRun) : 0u) | (LF_EPI_ZERO ? 0u : (1u << kRowEmpty));
     int64_t warps = (a.n_rows + 31) / 32;
-    int grid = (int)std::max<int64_t>(1, std::min<int64_t>((warps + 7) / 8, 148LL * 16));
+    int grid = (int)std::max<int64_t>(1, std::min<int64_t>((warps + 7) / 8, (int64_t)sm_count() * 16));
     zero_rows_kernel<<<grid, 256, 0, s>>>(a.row_mode, a.n_rows, a.C, a.ldc, a.J, vec4, mask);
     return cudaGetLastError();
 }
@@ -1359,6 +1360,13 @@ bool grouped_ok(const SpmmArgs &a) {
 
 bool mma_ok(const SpmmArgs &a) {
     return a.mma && a.nb_g > 0 && vec4_ok(a.B, a.ldb, a.C, a.ldc, a.J) && a.J % 64 == 0 && a.J <= 128;
+}
+
+const char *cell_spmm_path(const SpmmArgs &a) {
+    if (a.J == 0 || a.n_rows == 0) return "";
+    if (mma_ok(a)) return "cell_spmm_mma_kernel";
+    if (grouped_ok(a)) return "cell_spmm_grouped_kernel";
+    return "cell_spmm_kernel";
 }
 
 cudaError_t launch_cell_spmm(const SpmmArgs &a, cudaStream_t s) {

@@ -426,16 +426,7 @@ __global__ void __launch_bounds__(kThreads) stats_cols_kernel(const uint32_t *__
     }
 }
 
-int num_sms() {
-    static int n = 0;
-    if (!n) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
-        if (n <= 0) n = 148;
-    }
-    return n;
-}
+int num_sms() { return sm_count(); }
 
 }  // namespace
 

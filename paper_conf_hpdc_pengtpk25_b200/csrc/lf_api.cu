@@ -6,6 +6,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <string>
+#include <mutex>
 #include <vector>
 
 #include "lf_internal.cuh"
@@ -26,6 +27,38 @@ lf_status fail(lf_status st, const std::string &why) {
     } while (0)
 
 // ---- memory -------------------------------------------------------------
+// Scratch (configure / build) and handles built without an lf_allocator come
+// from a PRIVATE stream-ordered pool per device (cudaMemPoolCreate), not the
+// device's default pool: its release threshold is raised so memory survives
+// the synchronisations inside configure / build (a re-map costs
+// milliseconds), but bounded, and no other cudaMallocAsync user of the
+// process is affected.
+constexpr uint64_t kPoolKeepBytes = uint64_t(512) << 20;
+cudaMemPool_t scratch_pool() {
+    static std::mutex mu;
+    static cudaMemPool_t pools[64] = {};
+    const int dev = lf::current_device();
+    std::lock_guard<std::mutex> g(mu);
+    if (!pools[dev]) {
+        cudaMemPoolProps pr{};
+        pr.allocType = cudaMemAllocationTypePinned;
+        pr.handleTypes = cudaMemHandleTypeNone;
+        pr.location.type = cudaMemLocationTypeDevice;
+        pr.location.id = dev;
+        cudaMemPool_t p = nullptr;
+        if (cudaMemPoolCreate(&p, &pr) != cudaSuccess) return nullptr;
+        uint64_t thr = kPoolKeepBytes;
+        cudaMemPoolSetAttribute(p, cudaMemPoolAttrReleaseThreshold, &thr);
+        pools[dev] = p;
+    }
+    return pools[dev];
+}
+cudaError_t pool_alloc(void **p, size_t bytes, cudaStream_t s) {
+    cudaMemPool_t pool = scratch_pool();
+    if (!pool) return cudaErrorMemoryAllocation;
+    return cudaMallocFromPoolAsync(p, bytes, pool, s);
+}
+
 struct Mem {
     const lf_allocator *al;
     cudaStream_t s;
@@ -34,7 +67,7 @@ struct Mem {
         bytes = (bytes + 255) & ~size_t(255);
         if (al && al->alloc) return al->alloc(al->ctx, bytes, s);
         void *p = nullptr;
-        if (cudaMallocAsync(&p, bytes, s) != cudaSuccess) return nullptr;
+        if (pool_alloc(&p, bytes, s) != cudaSuccess) return nullptr;
         return p;
     }
     void put(void *p, size_t bytes) {
@@ -60,22 +93,6 @@ struct Scratch {
     }
 };
 
-// The device's default stream-ordered pool (cudaMallocAsync, used for the
-// configure scratch and when no lf_allocator is given) returns memory to the
-// OS at every synchronisation unless its release threshold is raised; a
-// re-map costs milliseconds, so keep the pool's memory (once per device).
-void keep_default_pool() {
-    static bool done[64] = {};
-    int dev = 0;
-    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64 || done[dev]) return;
-    cudaMemPool_t pool;
-    if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
-        uint64_t thr = UINT64_MAX;
-        cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
-    }
-    done[dev] = true;
-}
-
 lf_status check_csr(const lf_csr *A) {
     if (!A) return fail(LF_ERR_INVALID_ARG, "A is NULL");
     if (A->n_rows < 0 || A->n_cols < 0 || A->nnz < 0) return fail(LF_ERR_INVALID_ARG, "negative size");
@@ -90,7 +107,7 @@ lf_status maybe_validate(const lf_csr *A, cudaStream_t s) {
     const char *v = std::getenv("LF_VALIDATE");
     if (!v || v[0] != '1' || A->n_rows == 0) return LF_OK;
     int *d_flag = nullptr;
-    LF_CUDA(cudaMallocAsync(&d_flag, sizeof(int), s));
+    LF_CUDA(pool_alloc(reinterpret_cast<void **>(&d_flag), sizeof(int), s));
     LF_CUDA(cudaMemsetAsync(d_flag, 0, sizeof(int), s));
     LF_CUDA(lf::launch_validate(*A, d_flag, s));
     int flag = 0;
@@ -144,6 +161,19 @@ int alg3(const int64_t *cost, int hi) {
     return lo;
 }
 
+// SpMM kernel arguments of a handle (the counter slot is set per launch)
+lf::SpmmArgs spmm_args(const lf_cell *h, const float *B, int64_t ldb, int32_t J, float *C, int64_t ldc) {
+    const int nb = (int)h->buckets.size();
+    lf::SpmmArgs a{h->d_buckets + nb, h->d_buckets + nb + h->nb_n, h->nb_n, h->nb_w, h->n_tasks_n, h->n_tasks_w,
+                   h->slots_n, h->slots_w, 0, h->row_mode, h->n_rows, h->run_bound, nullptr, h->col_ind, h->val,
+                   h->row_tag, B, ldb, C, ldc, J,
+                   h->d_buckets + nb + h->nb_n + h->nb_w, h->nb_g, h->grouped, h->n_groups,
+                   h->d_buckets + nb + h->nb_n + h->nb_w + h->nb_g, h->mma, h->n_groups_m};
+    if (const char *g = std::getenv("LF_GROUPED")) a.grouped = g[0] == '1';
+    if (const char *g = std::getenv("LF_MMA")) a.mma = g[0] == '1';
+    return a;
+}
+
 }  // namespace
 
 extern "C" {
@@ -182,7 +212,6 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
     cudaStream_t s = (cudaStream_t)stream;
     if (lf_status st = maybe_validate(A, s)) return st;
 
-    keep_default_pool();
     // pinned staging buffer (one per thread) so the copies back are plain DMAs
     thread_local lf::StatsDev *h_st = nullptr;
     if (!h_st) LF_CUDA(cudaMallocHost(&h_st, sizeof(lf::StatsDev)));
@@ -194,7 +223,7 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
         const size_t b_st = (st_bytes + 255) & ~size_t(255), b_mask = (words * 4 + 255) & ~size_t(255);
         const size_t b_t0 = A->n_rows > 0 ? lf::stats_scratch_bytes(A->n_rows, A->nnz, P) : 0;
         char *d = nullptr;
-        LF_CUDA(cudaMallocAsync(&d, b_st + b_mask + b_t0 + 256, s));
+        LF_CUDA(pool_alloc(reinterpret_cast<void **>(&d), b_st + b_mask + b_t0 + 256, s));
         lf::StatsDev *d_st = reinterpret_cast<lf::StatsDev *>(d);
         uint32_t *d_mask = words ? reinterpret_cast<uint32_t *>(d + b_st) : nullptr;
         uint8_t *d_t0 = b_t0 ? reinterpret_cast<uint8_t *>(d + b_st + b_mask) : nullptr;
@@ -226,7 +255,7 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
         } else {
             lf::StatsDev *d_f = nullptr;
             const size_t fb = lf::stats_bytes(0);
-            LF_CUDA(cudaMallocAsync(&d_f, fb, s));
+            LF_CUDA(pool_alloc(reinterpret_cast<void **>(&d_f), fb, s));
             LF_CUDA(cudaMemsetAsync(d_f, 0, fb, s));
             LF_CUDA(cudaMemsetAsync(&d_f->len_min, 0xFF, sizeof(unsigned long long), s));
             LF_CUDA(lf::launch_features(*A, d_f, s));
@@ -256,7 +285,7 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
     if (!have && !need_stats && !predict) {  // forced CSR: the features alone
         lf::StatsDev *d_f = nullptr;
         const size_t fb = lf::stats_bytes(0);
-        LF_CUDA(cudaMallocAsync(&d_f, fb, s));
+        LF_CUDA(pool_alloc(reinterpret_cast<void **>(&d_f), fb, s));
         LF_CUDA(cudaMemsetAsync(d_f, 0, fb, s));
         LF_CUDA(cudaMemsetAsync(&d_f->len_min, 0xFF, sizeof(unsigned long long), s));
         LF_CUDA(lf::launch_features(*A, d_f, s));
@@ -332,10 +361,26 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
             return fail(LF_ERR_INVALID_ARG, "need 0 <= e_p <= k_p <= 30");
     }
     if (al && (!al->alloc || !al->free)) return fail(LF_ERR_INVALID_ARG, "allocator without alloc/free");
-    if (stats && stats->n_parts != P) return fail(LF_ERR_INVALID_ARG, "stats were computed for another n_parts");
+    if (stats) {  // the bucket sizes come from the stats: they must describe THIS A at this P
+        if (stats->n_parts != P) return fail(LF_ERR_INVALID_ARG, "stats were computed for another n_parts");
+        if (stats->features[0] != (double)A->n_rows || stats->features[1] != (double)A->n_cols ||
+            stats->features[2] != (double)A->nnz)
+            return fail(LF_ERR_INVALID_ARG, "stats were computed for another matrix (n_rows / n_cols / nnz differ)");
+        // F[p][0] = sum of the segment lengths of partition p, so the F[.][0]
+        // column sums to nnz exactly; tables zeroed by a CSR-format configure
+        // (or a stale / foreign struct) fail this
+        int64_t f0 = 0;
+        for (int p = 0; p < P; p++) {
+            f0 += stats->F[p][0];
+            for (int t = 0; t < lf::kMaxT; t++)
+                if (stats->H[p][t] < 0 || stats->F[p][t] < 0) return fail(LF_ERR_INVALID_ARG, "negative stats table entry");
+        }
+        if (f0 != A->nnz)
+            return fail(LF_ERR_INVALID_ARG, "stats tables do not cover A (sum of F[p][0] != nnz): configure chose "
+                                            "the CSR format or the stats belong to another matrix");
+    }
     cudaStream_t s = (cudaStream_t)stream;
     if (lf_status st = maybe_validate(A, s)) return st;
-    keep_default_pool();
 
     lf_cell *h = new lf_cell();
     h->params = *params;
@@ -499,6 +544,14 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
     } else {
         bs.src_pos = reinterpret_cast<int64_t *>(scr + s_head);
         bs.src_cnt = reinterpret_cast<int32_t *>(scr + s_head + up((size_t)R_tot * 8));
+        const char *v = std::getenv("LF_VALIDATE");
+        if (v && v[0] == '1' && n_tiles > 0) {  // the GPU-counted bucket sizes must equal the stats' ones
+            std::vector<long long> cnt(tot.size(), 0);
+            if ((st = cu(cudaMemcpyAsync(cnt.data(), bs.key_total, cnt.size() * 8, cudaMemcpyDeviceToHost, s), "D2H")))
+                return bail(st);
+            if ((st = cu(cudaStreamSynchronize(s), "sync"))) return bail(st);
+            if (cnt != tot) return bail(fail(LF_ERR_INVALID_ARG, "bucket sizes counted on the GPU differ from the stats"));
+        }
     }
     const int nb = (int)h->buckets.size();
 
@@ -566,18 +619,52 @@ lf_status lf_spmm(const lf_cell *h, const float *B, int64_t ldb, int32_t J, floa
         LF_CUDA(lf::launch_csr_spmm(h->csr, B, ldb, J, C, ldc, s));
         return LF_OK;
     }
-    const int nb = (int)h->buckets.size();
-    lf::SpmmArgs a{h->d_buckets + nb, h->d_buckets + nb + h->nb_n, h->nb_n, h->nb_w, h->n_tasks_n, h->n_tasks_w,
-                   h->slots_n, h->slots_w, 0, h->row_mode, h->n_rows, h->run_bound,
-                   h->ctr_ring + 4 * (h->launch_seq.fetch_add(1, std::memory_order_relaxed) % kCtrSlots), h->col_ind, h->val,
-                   h->row_tag,
-                   B, ldb, C, ldc, J,
-                   h->d_buckets + nb + h->nb_n + h->nb_w, h->nb_g, h->grouped, h->n_groups,
-                   h->d_buckets + nb + h->nb_n + h->nb_w + h->nb_g, h->mma, h->n_groups_m};
-    if (const char *g = std::getenv("LF_GROUPED")) a.grouped = g[0] == '1';
-    if (const char *g = std::getenv("LF_MMA")) a.mma = g[0] == '1';
+    lf::SpmmArgs a = spmm_args(h, B, ldb, J, C, ldc);
+    const uint32_t k = h->launch_seq.fetch_add(1, std::memory_order_relaxed) % kCtrSlots;
+    a.ctr = h->ctr_ring + 4 * k;
+    std::lock_guard<std::mutex> g(h->mu);
+    if (s == h->stream && !h->multi) {  // the common case: one stream, launches ordered by it
+        LF_CUDA(lf::launch_cell_spmm(a, s));
+        return LF_OK;
+    }
+    // several streams: a counter slot whose previous launch ran on another
+    // stream is fenced behind it, and every stream's last launch is recorded
+    // for lf_cell_destroy
+    if (!h->multi) {  // every earlier launch ran on the build stream
+        h->multi = true;
+        for (int q = 0; q < kCtrSlots; q++) h->slot_stream[q] = h->stream;
+    }
+    if (h->slot_stream[k] != s) {
+        if (!h->slot_ev[k]) LF_CUDA(cudaEventCreateWithFlags(&h->slot_ev[k], cudaEventDisableTiming));
+        if (!h->slot_recorded[k])  // earlier launches of the build stream were not recorded
+            LF_CUDA(cudaEventRecord(h->slot_ev[k], h->stream));
+        LF_CUDA(cudaStreamWaitEvent(s, h->slot_ev[k], 0));
+    }
     LF_CUDA(lf::launch_cell_spmm(a, s));
+    if (!h->slot_ev[k]) LF_CUDA(cudaEventCreateWithFlags(&h->slot_ev[k], cudaEventDisableTiming));
+    LF_CUDA(cudaEventRecord(h->slot_ev[k], s));
+    h->slot_recorded[k] = true;
+    h->slot_stream[k] = s;
+    if (s != h->stream) {
+        cudaEvent_t *e = nullptr;
+        for (auto &x : h->ext)
+            if (x.first == s) e = &x.second;
+        if (!e) {
+            h->ext.push_back({s, nullptr});
+            e = &h->ext.back().second;
+            LF_CUDA(cudaEventCreateWithFlags(e, cudaEventDisableTiming));
+        }
+        LF_CUDA(cudaEventRecord(*e, s));
+    }
     return LF_OK;
+}
+
+const char *lf_spmm_kernel_name(const lf_cell *h, int32_t J) {
+    if (!h || J <= 0) return "";
+    if (h->params.use_cell == 0) return "csr_spmm_kernel";
+    static const float *kAligned = reinterpret_cast<const float *>(uintptr_t(256));
+    lf::SpmmArgs a = spmm_args(h, kAligned, J, J, const_cast<float *>(kAligned), J);
+    return lf::cell_spmm_path(a);
 }
 
 lf_status lf_csr_spmm(const lf_csr *A, const float *B, int64_t ldb, int32_t J, float *C, int64_t ldc,
@@ -610,6 +697,14 @@ lf_status lf_cell_view(const lf_cell *h, lf_cell_arrays *out) {
 
 lf_status lf_cell_destroy(lf_cell *h) {
     if (!h) return LF_OK;
+    // the free is ordered on the build stream: after every lf_spmm launched on
+    // another stream too (their last launches were recorded)
+    for (auto &x : h->ext) {
+        cudaStreamWaitEvent(h->stream, x.second, 0);
+        cudaEventDestroy(x.second);
+    }
+    for (int q = 0; q < kCtrSlots; q++)
+        if (h->slot_ev[q]) cudaEventDestroy(h->slot_ev[q]);
     Mem mem{h->custom_al ? &h->al : nullptr, h->stream};
     mem.put(h->pool, h->pool_bytes);
     delete h;

@@ -8,6 +8,7 @@
 
 #include <string>
 #include <atomic>
+#include <mutex>
 #include <vector>
 
 #include "liteform.h"
@@ -25,6 +26,25 @@ __host__ __device__ __forceinline__ int ceil_log2_i64(int64_t l) {
     while ((int64_t(1) << t) < l) t++;
     return t;
 #endif
+}
+
+// Multiprocessors of the current device (queried once per device; grids are
+// sized in multiples of it, never from a hardcoded 148).
+inline int sm_count() {
+    static std::atomic<int> cache[64];
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) dev = 0;
+    int n = cache[dev].load(std::memory_order_relaxed);
+    if (n <= 0) {
+        if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n <= 0) n = 1;
+        cache[dev].store(n, std::memory_order_relaxed);
+    }
+    return n;
+}
+inline int current_device() {
+    int dev = 0;
+    if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) dev = 0;
+    return dev;
 }
 
 // Per-bucket descriptor the SpMM kernel walks (device copy of the bucket
@@ -152,6 +172,8 @@ struct SpmmArgs {
     int64_t n_groups_m;
 };
 cudaError_t launch_cell_spmm(const SpmmArgs &a, cudaStream_t s);  // pre-zeroes kRowRed rows itself
+// name of the kernel launch_cell_spmm runs for these arguments
+const char *cell_spmm_path(const SpmmArgs &a);
 cudaError_t launch_csr_spmm(const lf_csr &A, const float *B, int64_t ldb, int J, float *C, int64_t ldc,
                             cudaStream_t s);
 cudaError_t launch_validate(const lf_csr &A, int *d_flag, cudaStream_t s);
@@ -191,4 +213,13 @@ struct lf_cell {
     bool custom_al = false;
     cudaStream_t stream = nullptr;
     lf_csr csr{};  // use_cell == 0: the caller's CSR (must outlive the handle)
+    // lf_spmm on streams other than the build stream (lf_api.cu): each such
+    // stream's last launch is recorded so lf_cell_destroy orders the free
+    // after it, and counter slots reused across streams are fenced
+    mutable std::mutex mu;
+    mutable bool multi = false;
+    mutable std::vector<std::pair<cudaStream_t, cudaEvent_t>> ext;
+    mutable cudaEvent_t slot_ev[kCtrSlots] = {};
+    mutable cudaStream_t slot_stream[kCtrSlots] = {};
+    mutable bool slot_recorded[kCtrSlots] = {};
 };

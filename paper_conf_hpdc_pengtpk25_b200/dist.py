@@ -87,24 +87,26 @@ def col_bounds(J: int, world: int, align: int = 4) -> np.ndarray:
 
 
 def gather_cols(C_slab: torch.Tensor, cbounds, group=None) -> torch.Tensor:
-    """All-gather column slabs [I, J_r] into the full [I, J] C (one
-    all_gather of the padded slabs, then one strided copy per slab)."""
+    """All-gather column slabs [I, J_r] into the full [I, J] C: one
+    all_gather of the slabs (padded only when the slabs differ in width) and
+    ONE permuting copy [world, I, w] -> [I, world * w] into C."""
     world = dist.get_world_size(group)
     cb = [int(x) for x in cbounds]
-    wmax = max(cb[r + 1] - cb[r] for r in range(world))
+    widths = [cb[r + 1] - cb[r] for r in range(world)]
+    wmax = max(widths)
     I = C_slab.shape[0]
-    pad = torch.zeros((I, wmax), dtype=C_slab.dtype, device=C_slab.device)
-    pad[:, :C_slab.shape[1]] = C_slab
+    equal = all(w == wmax for w in widths)
+    src = C_slab.contiguous() if equal else torch.nn.functional.pad(C_slab, (0, wmax - C_slab.shape[1]))
+    buf = torch.empty((world, I, wmax), dtype=C_slab.dtype, device=C_slab.device)
     if dist.get_backend(group) == "nccl":
-        buf = torch.empty((world, I, wmax), dtype=C_slab.dtype, device=C_slab.device)
-        dist.all_gather_into_tensor(buf, pad, group=group)
-        parts = [buf[r] for r in range(world)]
+        dist.all_gather_into_tensor(buf, src, group=group)
     else:
-        parts = [torch.empty_like(pad) for _ in range(world)]
-        dist.all_gather(parts, pad, group=group)
+        dist.all_gather(list(buf.unbind(0)), src, group=group)
+    if equal:
+        return buf.permute(1, 0, 2).reshape(I, cb[-1])
     C = torch.empty((I, cb[-1]), dtype=C_slab.dtype, device=C_slab.device)
     for r in range(world):
-        C[:, cb[r]:cb[r + 1]] = parts[r][:, :cb[r + 1] - cb[r]]
+        C[:, cb[r]:cb[r + 1]] = buf[r, :, :widths[r]]
     return C
 
 

@@ -39,11 +39,14 @@ def _worker(rank, world, port, mode, q):
         full, _ = oracle.spmm_csr(A, B, with_abs=False)
         ok = bool(np.array_equal(C.numpy(), full))
         # large-J mode: column slabs of B, each rank's slab of C, gathered
-        cb = lfd.col_bounds(J, world)
-        j0, j1 = int(cb[rank]), int(cb[rank + 1])
-        C_slab, _ = oracle.spmm_csr(A, np.ascontiguousarray(B[:, j0:j1]), with_abs=False)
-        Cc = lfd.gather_cols(torch.from_numpy(C_slab.astype(np.float64)), cb)
-        ok = ok and bool(np.array_equal(Cc.numpy(), full))
+        for Jc in (J, 26):  # equal slabs (one permuting copy) and unequal ones (12 + 14: padded)
+            Bc = gen.dense(A.n_cols, Jc, 3, gen.INT, -15, 15)
+            fullc, _ = oracle.spmm_csr(A, Bc, with_abs=False)
+            cb = lfd.col_bounds(Jc, world)
+            j0, j1 = int(cb[rank]), int(cb[rank + 1])
+            C_slab, _ = oracle.spmm_csr(A, np.ascontiguousarray(Bc[:, j0:j1]), with_abs=False)
+            Cc = lfd.gather_cols(torch.from_numpy(C_slab.astype(np.float64)), cb)
+            ok = ok and bool(np.array_equal(Cc.numpy(), fullc))
         q.put((rank, ok, bounds.tolist()))
     finally:
         dist.destroy_process_group()

@@ -258,18 +258,105 @@ def test_full_config_parity(lf, name):
 
 
 def test_full_reddit_parity(lf):
+    """c4 (Reddit-shaped, 114.6M nnz) on its production path: the predictor's P
+    (8 on B200), widths from the GPU statistics.  The widths must equal the
+    oracle's Algorithm 3 per partition, the WHOLE CELL (every array, every
+    bucket) must equal the oracle's bit for bit, and sampled C rows (incl. the
+    20 longest) must be within tolerance."""
     A_h, J = gen.config("c4_reddit")
     A = lf.Csr.from_host(A_h)
-    params, _ = lf.configure(A, J)
-    M = lf.CellMatrix.build(A, params)
+    params, stats = lf.configure(A, J)
+    P = params.n_parts
+    assert params.use_cell == 1
+    e_or, _ = oracle.configure(A_h, P, J)
+    assert list(params.max_width_log2[:P]) == e_or.tolist()
+    M = lf.CellMatrix.build(A, params, stats)  # bench path: sizes from the stats, no sync
+    cell = oracle.csr_to_cell(A_h, P, list(params.max_width_log2[:P]), list(params.block_nnz_log2[:P]))
+    assert_cell_equal(M, cell)
+    del cell
     B_h = gen.dense(A_h.n_cols, J, 0)
     rng = np.random.default_rng(1)
     l = A_h.row_lengths()
     rows = np.unique(np.concatenate([rng.integers(0, A_h.n_rows, 500), np.argsort(l)[-20:]])).astype(np.int64)
     spmm_check(M, A_h, B_h, rows=rows)
-    # builder: the arrays of the 20 longest rows' buckets via the round-trip
-    v = M.view()
-    assert int(v["n_slots"]) >= A_h.nnz
+
+
+def test_reddit_shard_p8(lf):
+    """A 1/8 row shard of c4 (the multi-GPU unit of work, nnz-balanced bounds)
+    configured and built from a row_ptr VIEW with a non-zero base at P = 8:
+    configure == the oracle's Algorithm 3 on the standalone sub-CSR, CELL bit-exact,
+    C exact on integer inputs."""
+    from paper_conf_hpdc_pengtpk25_b200 import dist as lfd
+    A_h, J = gen.config("c4_reddit", kind=gen.INT, lo=-3, hi=3)
+    bounds = lfd.shard_bounds(A_h.row_ptr, 8, J, "nnz")
+    lo, hi = int(bounds[3]), int(bounds[4])
+    p0, p1 = int(A_h.row_ptr[lo]), int(A_h.row_ptr[hi])
+    sub = gen.CSR(hi - lo, A_h.n_cols, A_h.row_ptr[lo:hi + 1] - p0, A_h.col_ind[p0:p1], A_h.val[p0:p1])
+    A = lf.Csr.from_host(A_h)
+    shard = lf.Csr(A.row_ptr[lo:hi + 1], A.col_ind, A.val, A.n_cols, p1 - p0)
+    params, stats = lf.configure(shard, J, force_parts=8, force_format=1)
+    e_or, _ = oracle.configure(sub, 8, J)
+    assert list(params.max_width_log2[:8]) == e_or.tolist()
+    for p in range(8):
+        top = oracle.partition_max_log2(sub, 8, p)
+        assert stats.max_log2[p] == top
+        for e in range(max(0, e_or[p] - 1), min(top, e_or[p] + 1) + 1):
+            assert stats.cost[p][e] == oracle.partition_cost(sub, 8, p, e, J)
+    M = lf.CellMatrix.build(shard, params, stats)
+    assert_cell_equal(M, oracle.csr_to_cell(sub, 8, list(params.max_width_log2[:8]),
+                                            list(params.block_nnz_log2[:8])))
+    B_h = gen.dense(A_h.n_cols, J, 5, gen.INT, -15, 15)
+    rng = np.random.default_rng(2)
+    rows = np.unique(np.concatenate([rng.integers(0, sub.n_rows, 400),
+                                     np.argsort(sub.row_lengths())[-10:]])).astype(np.int64)
+    spmm_check(M, sub, B_h, exact=True, rows=rows)
+
+
+@pytest.mark.parametrize("name", ["c2_rmat20", "c3_stencil126", "c3b_banded2M"])
+def test_full_configure_matches_oracle(lf, name):
+    """Full-size configure (nnz > 2^25 takes the features-first path on c3 /
+    c3b) against the oracle at the P the predictor chose: every eq. 7 cost of
+    every partition, the statistics tables (P = 1) and Algorithm 3's e_p."""
+    A_h, J = gen.config(name)
+    A = lf.Csr.from_host(A_h)
+    for Jx in (J, 128):
+        params, st = lf.configure(A, Jx, force_format=1)
+        P = params.n_parts
+        e_or, k_or = oracle.configure(A_h, P, Jx)
+        assert list(params.max_width_log2[:P]) == e_or.tolist()
+        assert list(params.block_nnz_log2[:P]) == k_or.tolist()
+        for p in range(P):
+            top = oracle.partition_max_log2(A_h, P, p)
+            assert st.max_log2[p] == top
+            assert [st.cost[p][e] for e in range(top + 1)] == \
+                [oracle.partition_cost(A_h, P, p, e, Jx) for e in range(top + 1)]
+            if P == 1 and Jx == J:
+                H, F, Un, Ut = oracle.partition_stats(A_h, P, p)
+                assert list(st.H[p]) == H.tolist() and list(st.F[p]) == F.tolist()
+                assert list(st.Unat[p]) == Un.tolist() and list(st.Utop[p]) == Ut.tolist()
+
+
+@pytest.mark.parametrize("P", [6, 7, 8])
+@pytest.mark.parametrize("seed", range(4))
+def test_builder_bit_exact_many_parts(lf, P, seed):
+    """P >= 6 (c4's production P is 8): random widths and block multipliers on
+    random CSR with duplicates / explicit zeros, and configure-chosen widths on
+    an R-MAT, both bit-exact; integer SpMM exact."""
+    rng = np.random.default_rng(500 + 10 * P + seed)
+    A_h = gen.random_small(int(rng.integers(50, 400)), int(rng.integers(P, 300)), 120, seed, dup=True, zeros=True,
+                           kind=gen.INT, lo=-3, hi=3)
+    e = rng.integers(0, 7, size=P).tolist()
+    k = [x + int(rng.integers(0, 3)) for x in e]
+    _, M = build(lf, A_h, P, e, k)
+    assert_cell_equal(M, oracle.csr_to_cell(A_h, P, e, k))
+    spmm_check(M, A_h, gen.dense(A_h.n_cols, 64, seed, gen.INT, -15, 15), exact=True)
+    R_h = gen.rmat(12, 16, seed=seed, kind=gen.INT, lo=-3, hi=3)
+    R = lf.Csr.from_host(R_h)
+    params, stats = lf.configure(R, 128, force_parts=P, force_format=1)
+    M2 = lf.CellMatrix.build(R, params, stats)
+    assert_cell_equal(M2, oracle.csr_to_cell(R_h, P, list(params.max_width_log2[:P]),
+                                             list(params.block_nnz_log2[:P])))
+    spmm_check(M2, R_h, gen.dense(R_h.n_cols, 128, seed, gen.INT, -15, 15), exact=True)
 
 
 @pytest.mark.parametrize("width", [None, 12])
@@ -367,3 +454,64 @@ def test_steps_in_flight_on_lanes(lf, n_lanes):
     torch.cuda.synchronize()
     for C in got:
         assert np.array_equal(C.cpu().numpy().astype(np.float64), ref)
+
+
+def test_build_rejects_foreign_stats(lf):
+    """lf_cell_build sizes its arrays from the stats, so it must refuse stats of
+    another matrix (same P), stats of a CSR-format configure (tables zeroed)
+    and stats whose tables were tampered with -- an error, never an
+    out-of-bounds write."""
+    A_h = gen.rmat(11, 16, seed=1)
+    B_h = gen.rmat(11, 8, seed=2)
+    A, Bm = lf.Csr.from_host(A_h), lf.Csr.from_host(B_h)
+    pa, sa = lf.configure(A, 64, force_parts=2, force_format=1)
+    _, sb = lf.configure(Bm, 64, force_parts=2, force_format=1)
+    with pytest.raises(lf.LfError):
+        lf.CellMatrix.build(A, pa, sb)  # another matrix
+    _, scsr = lf.configure(A, 64, force_parts=2, force_format=2)
+    with pytest.raises(lf.LfError):
+        lf.CellMatrix.build(A, pa, scsr)  # CSR format: no tables
+    sa.F[0][0] -= 1
+    with pytest.raises(lf.LfError):
+        lf.CellMatrix.build(A, pa, sa)  # tables do not cover A
+    sa.F[0][0] += 1
+    M = lf.CellMatrix.build(A, pa, sa)
+    assert_cell_equal(M, oracle.csr_to_cell(A_h, 2, list(pa.max_width_log2[:2]), list(pa.block_nnz_log2[:2])))
+
+
+def test_destroy_after_spmm_on_other_stream(lf):
+    """lf_spmm on a second stream, then close() right away: the free is ordered
+    (through the recorded event) after that launch, so memory the build stream
+    reuses and overwrites immediately cannot corrupt the running SpMM."""
+    A_h = gen.rmat(16, 16, seed=5, kind=gen.INT, lo=-3, hi=3)
+    B_h = gen.dense(A_h.n_cols, 128, 5, gen.INT, -15, 15)
+    A = lf.Csr.from_host(A_h)
+    B = torch.from_numpy(B_h).cuda()
+    ref = oracle.spmm_csr(A_h, B_h)[0]
+    s2 = torch.cuda.Stream()
+    for it in range(3):
+        params, stats = lf.configure(A, 128)
+        M = lf.CellMatrix.build(A, params, stats)  # build stream = current stream
+        torch.cuda.current_stream().synchronize()
+        s2.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.stream(s2):
+            C = M.spmm(B, stream=s2)
+        M.close()
+        junk = torch.full((64 << 20,), -7.0, device="cuda")  # reuses the freed pool on the build stream
+        del junk
+        s2.synchronize()
+        assert np.array_equal(C.cpu().numpy().astype(np.float64), ref)
+
+
+def test_kernel_name(lf):
+    A_h = gen.banded(4096, 12, seed=0)
+    A = lf.Csr.from_host(A_h)
+    p, s = lf.configure(A, 64, force_format=1)
+    M = lf.CellMatrix.build(A, p, s)
+    assert M.path(64) in ("cell_spmm_grouped_kernel", "cell_spmm_tc_kernel")
+    R_h = gen.rmat(12, 16, seed=0)
+    R = lf.Csr.from_host(R_h)
+    p, s = lf.configure(R, 128, force_format=1)
+    assert lf.CellMatrix.build(R, p, s).path(128) == "cell_spmm_kernel"
+    p, s = lf.configure(R, 128, force_format=2)
+    assert lf.CellMatrix.build(R, p, s).path(128) == "csr_spmm_kernel"
