@@ -150,7 +150,9 @@ typedef struct lf_configure_stats {
     int64_t cost[LF_MAX_PARTS][32];
     double group_union_ratio; /* sampled: distinct columns / nonzeros of groups of 4 consecutive rows */
     int32_t spmm_grouped;     /* 1: lf_cell_build given these stats makes lf_spmm take the grouped path */
-    int32_t pad_;
+    int32_t spmm_tc;          /* 1: ... the tcgen05 windowed path (32 <= J <= 128) */
+    double window_span_mean;  /* sampled groups of 128 consecutive rows: mean span (max - min column + 1) */
+    double window_over_frac;  /* ... fraction of sampled groups whose span exceeds 256 B rows */
 } lf_configure_stats;
 
 /* One CELL bucket (Fig. 4).  Buckets are stored
@@ -229,9 +231,11 @@ LF_API lf_status lf_predict(const double features[8], int32_t max_parts, int32_t
  *           from them (bucket t < e_p holds H[p][t] rows, the max bucket
  *           F[p][e_p]), so the build enqueues everything asynchronously with
  *           no host synchronisation.  NULL: the sizes are counted on the GPU
- *           and s is synchronised once.  stats->spmm_grouped = 1 makes the
- *           handle's lf_spmm take the grouped path (LF_GROUPED=0/1 in the
- *           environment overrides it per call).
+ *           and s is synchronised once.  stats->spmm_tc = 1 makes the
+ *           handle's lf_spmm take the tcgen05 windowed path (the per-group
+ *           B-row windows are built here), else stats->spmm_grouped = 1 the
+ *           grouped path (LF_TC=0/1 and LF_GROUPED=0/1 in the environment
+ *           override them; LF_TC=1 at build time builds the windows).
  * The handle may be used on s immediately.
  * Errors: LF_ERR_INVALID_ARG (sizes, e_p > k_p, P out of range; stats for a
  *         different P, for a matrix with other n_rows / n_cols / nnz, or with

@@ -63,7 +63,8 @@ class LfConfigureStats(ctypes.Structure):
     _fields_ = [("features", ctypes.c_double * 8), ("n_parts", _I32), ("max_log2", _I32 * LF_MAX_PARTS),
                 ("chosen_log2", _I32 * LF_MAX_PARTS), ("H", _T32 * LF_MAX_PARTS), ("F", _T32 * LF_MAX_PARTS),
                 ("Unat", _T32 * LF_MAX_PARTS), ("Utop", _T32 * LF_MAX_PARTS), ("cost", _T32 * LF_MAX_PARTS),
-                ("group_union_ratio", ctypes.c_double), ("spmm_grouped", _I32), ("pad_", _I32)]
+                ("group_union_ratio", ctypes.c_double), ("spmm_grouped", _I32), ("spmm_tc", _I32),
+                ("window_span_mean", ctypes.c_double), ("window_over_frac", ctypes.c_double)]
 
 
 class LfBucket(ctypes.Structure):

@@ -205,7 +205,7 @@ __global__ void __launch_bounds__(1024) tile_scan_kernel(long long *__restrict__
 // one block per bucket: its block-padding rows, and (block 0) the counters
 __global__ void pad_init_kernel(const BucketDev *__restrict__ bk, int nb, int32_t *__restrict__ row_ind,
                                 int32_t *__restrict__ row_tag, int32_t *__restrict__ src_cnt,
-                                unsigned long long *__restrict__ ctr, int n_ctr) {
+                                int64_t *__restrict__ src_pos, unsigned long long *__restrict__ ctr, int n_ctr) {
     if (blockIdx.x == 0)
         for (int q = threadIdx.x; q < n_ctr; q += blockDim.x) ctr[q] = 0;
     if ((int)blockIdx.x >= nb) return;
@@ -214,6 +214,7 @@ __global__ void pad_init_kernel(const BucketDev *__restrict__ bk, int nb, int32_
         row_ind[r] = -1;
         row_tag[r] = -1;
         src_cnt[r] = 0;
+        src_pos[r] = 0;  // never dereferenced (count 0), but defined (initcheck)
     }
 }
 
@@ -393,8 +394,8 @@ cudaError_t launch_tile_scan(int P, const BuildScratch &sc, cudaStream_t s) {
 }
 
 cudaError_t launch_pad_init(const BucketDev *bk, int nb, int32_t *row_ind, int32_t *row_tag, int32_t *src_cnt,
-                            unsigned long long *ctr, int n_ctr, cudaStream_t s) {
-    pad_init_kernel<<<std::max(nb, 1), 256, 0, s>>>(bk, nb, row_ind, row_tag, src_cnt, ctr, n_ctr);
+                            int64_t *src_pos, unsigned long long *ctr, int n_ctr, cudaStream_t s) {
+    pad_init_kernel<<<std::max(nb, 1), 256, 0, s>>>(bk, nb, row_ind, row_tag, src_cnt, src_pos, ctr, n_ctr);
     return cudaGetLastError();
 }
 

@@ -1364,6 +1364,7 @@ bool mma_ok(const SpmmArgs &a) {
 
 const char *cell_spmm_path(const SpmmArgs &a) {
     if (a.J == 0 || a.n_rows == 0) return "";
+    if (tc_ok(a)) return "cell_spmm_tc_kernel";
     if (mma_ok(a)) return "cell_spmm_mma_kernel";
     if (grouped_ok(a)) return "cell_spmm_grouped_kernel";
     return "cell_spmm_kernel";
@@ -1372,6 +1373,11 @@ const char *cell_spmm_path(const SpmmArgs &a) {
 cudaError_t launch_cell_spmm(const SpmmArgs &a, cudaStream_t s) {
     if (a.J == 0 || a.n_rows == 0) return cudaSuccess;
     const bool v4 = vec4_ok(a.B, a.ldb, a.C, a.ldc, a.J);
+    if (tc_ok(a)) {  // runs of folded rows are split across groups: red.add, pre-zeroed
+        cudaError_t e = zero_red_rows(a, true, s);
+        if (e != cudaSuccess) return e;
+        return launch_cell_spmm_tc(a, s);
+    }
     if (mma_ok(a)) {
         cudaError_t e = zero_red_rows(a, true, s);
         if (e != cudaSuccess) return e;

@@ -455,8 +455,38 @@ __global__ void __launch_bounds__(256) group_sample_kernel(const int64_t *__rest
     for (int q = lane; q < 256; q += 32) hs[w][q] = -1;
     __syncwarp();
     const int64_t smp = (int64_t)blockIdx.x * 8 + w;
+    if (smp >= kGroupSamples) return;
+    // tcgen05 windowed path (cell_spmm_tc.cu): the B-row window of 128
+    // consecutive rows = [min first column, max last column]; rows longer than
+    // 32 make the sample ineligible (the path needs every W <= 32)
+    {
+        const int64_t n_wg = n_rows / 128;
+        if (n_wg > 0) {
+            const int64_t i0 = (smp * n_wg / kGroupSamples) * 128;
+            const int64_t base0 = row_ptr[0];
+            int mn = INT32_MAX, mx = -1;
+            bool ok = true;
+            for (int r = lane; r < 128; r += 32) {
+                const int64_t b = row_ptr[i0 + r] - base0, e = row_ptr[i0 + r + 1] - base0;
+                ok = ok && e - b <= 32;
+                if (e > b) {
+                    mn = min(mn, col[base0 + b]);
+                    mx = max(mx, col[base0 + e - 1]);
+                }
+            }
+            ok = __all_sync(kFull, ok);
+            mn = __reduce_min_sync(kFull, mn);
+            mx = __reduce_max_sync(kFull, mx);
+            if (lane == 0 && ok && mx >= 0) {
+                const unsigned long long span = (unsigned long long)(mx - mn + 1);
+                atomicAdd(&st->win_span, span);
+                atomicAdd(&st->win_cnt, 1ull);
+                if (span > 256) atomicAdd(&st->win_over, 1ull);
+            }
+        }
+    }
     const int64_t n_groups = n_rows / kGroupRows;
-    if (smp >= kGroupSamples || n_groups == 0) return;
+    if (n_groups == 0) return;
     const int64_t i0 = (smp * n_groups / kGroupSamples) * kGroupRows;
     const int64_t base = row_ptr[0];
     int64_t b[kGroupRows], l[kGroupRows];

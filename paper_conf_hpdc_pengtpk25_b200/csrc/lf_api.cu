@@ -140,6 +140,8 @@ void table2_features(const lf_csr &A, int32_t J, const lf::StatsDev &st, double 
 // banded hw 4/8/12 (ratio 0.33-0.28) 1.06-1.8x faster, 32-wide dense blocks
 // (0.25) 1.8-2.0x, 27-point stencil (0.50) 1.2x; slower on R-MAT (0.96),
 // lognormal (~1), uniform (1.0, equal at J = 128) and rows of 8 (0.25, mean 8).
+constexpr double kTcMaxSpan = 256.0;   // mean sampled window (B rows per 128-row group)
+constexpr double kTcMaxOver = 0.02;    // sampled groups whose window exceeds the kernel's cap
 constexpr double kGroupedMaxRatio = 0.6;    // distinct columns / nonzeros of 4-row groups
 constexpr double kGroupedMinMeanLen = 8.5;  // mean row length
 double group_ratio(const lf::StatsDev &st) {
@@ -168,8 +170,10 @@ lf::SpmmArgs spmm_args(const lf_cell *h, const float *B, int64_t ldb, int32_t J,
                    h->slots_n, h->slots_w, 0, h->row_mode, h->n_rows, h->run_bound, nullptr, h->col_ind, h->val,
                    h->row_tag, B, ldb, C, ldc, J,
                    h->d_buckets + nb + h->nb_n + h->nb_w, h->nb_g, h->grouped, h->n_groups,
-                   h->d_buckets + nb + h->nb_n + h->nb_w + h->nb_g, h->mma, h->n_groups_m};
+                   h->d_buckets + nb + h->nb_n + h->nb_w + h->nb_g, h->mma, h->n_groups_m,
+                   h->d_buckets + nb + h->nb_n + h->nb_w + 2 * h->nb_g, h->nb_g, h->tc, h->n_groups_t, h->tc_win};
     if (const char *g = std::getenv("LF_GROUPED")) a.grouped = g[0] == '1';
+    if (const char *g = std::getenv("LF_TC")) a.tc = g[0] == '1';
     if (const char *g = std::getenv("LF_MMA")) a.mma = g[0] == '1';
     return a;
 }
@@ -342,6 +346,16 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
     bool narrow = true;
     for (int p = 0; p < P; p++) narrow = narrow && prm.max_width_log2[p] <= 5;
     cs.spmm_grouped = (use_cell && narrow && grouped_candidate(st, *A, J)) ? 1 : 0;
+    // tcgen05 windowed path (cell_spmm_tc.cu): groups of 128 rows whose
+    // columns fit a window of <= 256 B rows, the window short enough that
+    // the dense contraction (3 MMAs per 8 window rows) stays under the group's
+    // memory time; decided from the sampled windows
+    cs.window_span_mean = st.win_cnt ? (double)st.win_span / (double)st.win_cnt : 0.0;
+    cs.window_over_frac = st.win_cnt ? (double)st.win_over / (double)st.win_cnt : 1.0;
+    cs.spmm_tc = (use_cell && narrow && J >= 32 && J <= 128 && st.win_cnt > 0 && cs.window_over_frac <= kTcMaxOver &&
+                  cs.window_span_mean <= kTcMaxSpan)
+                     ? 1
+                     : 0;
     *out = prm;
     return LF_OK;
 }
@@ -385,6 +399,7 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
     lf_cell *h = new lf_cell();
     h->params = *params;
     h->grouped = stats ? stats->spmm_grouped : 0;
+    h->tc = stats ? stats->spmm_tc : 0;
     h->n_rows = A->n_rows;
     h->n_cols = A->n_cols;
     h->nnz = A->nnz;
@@ -488,6 +503,12 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
                 h->n_groups_m += (d.n_rows_pad + 15) / 16;
                 h->h_buckets.push_back(d);
             }
+            for (int q = 0; q < nb_all; q++) {  // and for 128-row groups (tcgen05 windowed path)
+                lf::BucketDev d = h->h_buckets[q];
+                d.task_off = h->n_groups_t;
+                h->n_groups_t += (d.n_rows_pad + lf::kTcGroupRows - 1) / lf::kTcGroupRows;
+                h->h_buckets.push_back(d);
+            }
             h->nb_g = nb_all;
         }
         if (h->buckets.size() > 2048) return fail(LF_ERR_UNSUPPORTED, "more than 2048 buckets");
@@ -562,7 +583,13 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
                  b_ri = up(R_tot * 4), b_rt = up(R_tot * 4), b_ci = up(S_tot * 4), b_va = up(S_tot * 4),
                  b_rb = up((size_t)(h->n_tasks_w + 1)), b_ct = up(kCtrSlots * 4 * sizeof(unsigned long long)),
                  b_rm = up((size_t)std::max<int64_t>(I, 1));
-    h->pool_bytes = b_bk + b_ko + b_ri + b_rt + b_ci + b_va + b_rb + b_ct + b_rm;
+    // tcgen05 windowed path: a window per 128-row group, built when configure
+    // chose the path (or LF_TC=1 asks for it, or the sizes are GPU-counted)
+    const char *tc_env = std::getenv("LF_TC");
+    const bool want_tc = h->nb_g > 0 && h->n_groups_t > 0 &&
+                         (tc_env ? tc_env[0] == '1' : (stats ? stats->spmm_tc != 0 : true));
+    const size_t b_tw = want_tc ? up((size_t)h->n_groups_t * sizeof(int2)) : 0;
+    h->pool_bytes = b_bk + b_ko + b_ri + b_rt + b_ci + b_va + b_rb + b_ct + b_rm + b_tw;
     h->pool = mem.get(h->pool_bytes);
     if (!h->pool) return bail(fail(LF_ERR_NO_MEMORY, "CELL arrays allocation failed"));
     char *q = static_cast<char *>(h->pool);
@@ -576,6 +603,7 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
     h->run_bound = reinterpret_cast<uint8_t *>(q + b_ri + b_rt + b_ci + b_va);
     h->ctr_ring = reinterpret_cast<unsigned long long *>(q + b_ri + b_rt + b_ci + b_va + b_rb);
     h->row_mode = reinterpret_cast<uint8_t *>(q + b_ri + b_rt + b_ci + b_va + b_rb + b_ct);
+    h->tc_win = b_tw ? reinterpret_cast<int2 *>(q + b_ri + b_rt + b_ci + b_va + b_rb + b_ct + b_rm) : nullptr;
     {
         std::vector<char> head(b_bk + b_ko, 0);
         if (!h->h_buckets.empty())
@@ -588,7 +616,7 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
     if (P > 1 && I > 0 && (st = cu(cudaMemsetAsync(h->row_mode, lf::kRowEmpty, (size_t)I, s), "memset")))
         return bail(st);
     // queue counters zero; padding rows' rowInd / tags -1 and src_cnt 0
-    if ((st = cu(lf::launch_pad_init(h->d_buckets, nb, h->row_ind, h->row_tag, bs.src_cnt, h->ctr_ring,
+    if ((st = cu(lf::launch_pad_init(h->d_buckets, nb, h->row_ind, h->row_tag, bs.src_cnt, bs.src_pos, h->ctr_ring,
                                      kCtrSlots * 4, s),
                  "pad_init")))
         return bail(st);
@@ -601,6 +629,11 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
     if ((st = cu(lf::launch_run_bounds(h->d_buckets + nb + h->nb_n, h->nb_w, h->n_tasks_w, h->row_tag, h->run_bound,
                                        s),
                  "run_bounds")))
+        return bail(st);
+    if (h->tc_win &&
+        (st = cu(lf::launch_tc_windows(h->d_buckets + nb + h->nb_n + h->nb_w + 2 * h->nb_g, h->nb_g, h->n_groups_t,
+                                       h->col_ind, bs.src_cnt, h->tc_win, s),
+                 "tc_windows")))
         return bail(st);
     *out = h;
     return LF_OK;

@@ -73,6 +73,7 @@ struct StatsPart {
 struct StatsDev {
     unsigned long long len_min, len_max, len_sum, len_sumsq;  // row lengths
     unsigned long long grp_union, grp_nnz;  // sampled groups of kGroupRows rows: distinct columns, nonzeros
+    unsigned long long win_span, win_cnt, win_over;  // sampled groups of 128 rows: summed spans, samples, spans > 256
     StatsPart part[LF_MAX_PARTS];  // only the first P are cleared / copied back
 };
 inline size_t stats_bytes(int P) { return offsetof(StatsDev, part) + (size_t)P * sizeof(StatsPart); }
@@ -131,7 +132,7 @@ cudaError_t launch_bucket_count(const lf_csr &A, int P, const WidthArg &e, const
 // padding rows (n_real_rows .. n_rows_pad of every bucket): rowInd / tag -1,
 // src_cnt 0; and the n_ctr queue counters zeroed
 cudaError_t launch_pad_init(const BucketDev *bk, int nb, int32_t *row_ind, int32_t *row_tag, int32_t *src_cnt,
-                            unsigned long long *ctr, int n_ctr, cudaStream_t s);
+                            int64_t *src_pos, unsigned long long *ctr, int n_ctr, cudaStream_t s);
 cudaError_t launch_tile_scan(int P, const BuildScratch &sc, cudaStream_t s);
 cudaError_t launch_bucket_place(const lf_csr &A, int P, const WidthArg &e, const BuildScratch &sc,
                                 const int32_t *row_cnt, int32_t *row_ind, int32_t *row_tag, uint8_t *row_mode,
@@ -170,10 +171,23 @@ struct SpmmArgs {
     const BucketDev *bk_m;
     int mma;
     int64_t n_groups_m;
+    // tcgen05 windowed path (cell_spmm_tc.cu): the same buckets, task_off
+    // counting 128-row groups, and each group's B-row window {lo, span}
+    const BucketDev *bk_t;
+    int nb_t;
+    int tc;
+    int64_t n_groups_t;
+    const int2 *tc_win;
 };
 cudaError_t launch_cell_spmm(const SpmmArgs &a, cudaStream_t s);  // pre-zeroes kRowRed rows itself
 // name of the kernel launch_cell_spmm runs for these arguments
 const char *cell_spmm_path(const SpmmArgs &a);
+// tcgen05 windowed path (cell_spmm_tc.cu)
+constexpr int kTcGroupRows = 128;
+bool tc_ok(const SpmmArgs &a);
+cudaError_t launch_cell_spmm_tc(const SpmmArgs &a, cudaStream_t s);
+cudaError_t launch_tc_windows(const BucketDev *bk_t, int nb_t, int64_t n_groups, const int32_t *col,
+                              const int32_t *src_cnt, int2 *win, cudaStream_t s);
 cudaError_t launch_csr_spmm(const lf_csr &A, const float *B, int64_t ldb, int J, float *C, int64_t ldc,
                             cudaStream_t s);
 cudaError_t launch_validate(const lf_csr &A, int *d_flag, cudaStream_t s);
@@ -199,6 +213,9 @@ struct lf_cell {
     int grouped = 0;         // lf_spmm takes the grouped path
     int64_t n_groups_m = 0;  // 16-row groups (tensor-core grouped path)
     int mma = 0;             // lf_spmm takes the tensor-core grouped path
+    int64_t n_groups_t = 0;  // 128-row groups of the tcgen05 windowed path
+    int2 *tc_win = nullptr;  // [n_groups_t] B-row window per group (in the pool; NULL: not built)
+    int tc = 0;              // lf_spmm takes the tcgen05 windowed path
     // work-queue counters, kCtrSlots slots of 4 (wide, narrow, warps done, -)
     // in the pool: launch k uses slot k % kCtrSlots and its last warp resets
     // it, so lf_spmm needs no allocation or memset per call

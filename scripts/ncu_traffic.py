@@ -47,8 +47,8 @@ def measure(cfg, J):
         if r.get("Metric Name") in tot:
             v = float(r["Metric Value"].replace(",", ""))
             u = r.get("Metric Unit", "")
-            scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "nsecond": 1e-3, "usecond": 1,
-                     "msecond": 1e3}.get(u, 1)
+            scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "nsecond": 1e-3, "ns": 1e-3,
+                     "usecond": 1, "us": 1, "msecond": 1e3, "ms": 1e3}.get(u, 1)
             tot[r["Metric Name"]] += v * scale
             names.add(r["Kernel Name"].split("(")[0].split("<")[0])
     return {"kernels": sorted(names), "dram_read": int(tot["dram__bytes_read.sum"]),
