@@ -218,6 +218,25 @@ __device__ __forceinline__ TcGroup tc_group(const SpmmArgs &a, int64_t g, int &b
     return x;
 }
 
+// The CTA's groups g = blockIdx.x, + gridDim.x, ...; the NEXT group's
+// descriptor is fetched when a group starts, so its global loads (bucket
+// table, window) are in flight while the current group is processed instead
+// of stalling every role at every group boundary.
+struct TcIter {
+    int64_t g, n;
+    int bcur;
+    TcGroup x, nx;
+    __device__ __forceinline__ TcIter(const SpmmArgs &a) : g(blockIdx.x), n(a.n_groups_t), bcur(0) {
+        if (g < n) x = tc_group(a, g, bcur);
+        if (g + gridDim.x < n) nx = tc_group(a, g + gridDim.x, bcur);
+    }
+    __device__ __forceinline__ void next(const SpmmArgs &a) {
+        g += gridDim.x;
+        x = nx;
+        if (g + gridDim.x < n) nx = tc_group(a, g + gridDim.x, bcur);
+    }
+};
+
 __device__ __forceinline__ bool tag_whole(int32_t tag) { return (tag & 7) == 7; }
 __device__ __forceinline__ int32_t tag_row(int32_t tag) { return tag >> 3; }
 
@@ -327,7 +346,6 @@ __global__ void __launch_bounds__(kTcWarps * 32, 1) cell_spmm_tc_kernel(const Sp
     const uint32_t tmem = sm.tmem;
     const int64_t n_groups = a.n_groups_t;
     const uint64_t pol = policy_evict_first();
-    int bcur = 0;
 
     if (warp < kWEpi) {
         // ===== loaders: landed B window chunk (smem) -> TMEM A operand, raw + lo =====
@@ -335,8 +353,8 @@ __global__ void __launch_bounds__(kTcWarps * 32, 1) cell_spmm_tc_kernel(const Sp
         const bool jok = j < a.J;
         const uint32_t lane_base = tmem + ((uint32_t)(32 * warp) << 16);
         uint32_t sa = 0, pha = 0, sb = 0, phb = 0, mb = 0, phm = 0;
-        for (int64_t g = blockIdx.x; g < n_groups; g += gridDim.x) {
-            const TcGroup x = tc_group(a, g, bcur);
+        for (TcIter it(a); it.g < n_groups; it.next(a)) {
+            const TcGroup &x = it.x;
             if (!x.mma) continue;
             TC_WAIT(0, &sm.full_m[mb], phm);
             for (int c = 0; c < x.nch; c++) {
@@ -382,8 +400,8 @@ __global__ void __launch_bounds__(kTcWarps * 32, 1) cell_spmm_tc_kernel(const Sp
         const bool jok = j < a.J;
         const uint32_t lane_base = tmem + ((uint32_t)(32 * q) << 16);
         uint32_t d = 0, phd = 0;
-        for (int64_t g = blockIdx.x; g < n_groups; g += gridDim.x) {
-            const TcGroup x = tc_group(a, g, bcur);
+        for (TcIter it(a); it.g < n_groups; it.next(a)) {
+            const TcGroup &x = it.x;
             if (!x.mma) continue;
             int32_t tags[kTcN / 32];
 #pragma unroll
@@ -438,14 +456,11 @@ __global__ void __launch_bounds__(kTcWarps * 32, 1) cell_spmm_tc_kernel(const Sp
         const int bw = warp - kWBuild;
         zero_empty_rows(a, (int64_t)blockIdx.x * kNBuild + bw, (int64_t)gridDim.x * kNBuild, lane, pol);
         uint32_t sv = 0, phv = 0, mb = 0, phm = 0, sc = 0, phc = 0;
-        for (int64_t g = blockIdx.x; g < n_groups; g += gridDim.x) {
+        for (TcIter it(a); it.g < n_groups; it.next(a)) {
 #ifdef LF_TC_TRACE
             long long tb0 = clock64();
 #endif
-            const TcGroup x = tc_group(a, g, bcur);
-#ifdef LF_TC_TRACE
-            if (lane == 0) atomicAdd(&lf_tc_trace[blockIdx.x][18], (unsigned long long)(clock64() - tb0));
-#endif
+            const TcGroup &x = it.x;
             if (x.span == 0) continue;
             if (!x.mma) {
                 fallback_group(a, x, bw, lane, pol);
@@ -507,6 +522,21 @@ __global__ void __launch_bounds__(kTcWarps * 32, 1) cell_spmm_tc_kernel(const Sp
             if (lane == 0) mbar_arrive(&sm.full_m[mb]);
             mb ^= 1;
             if (mb == 0) phm ^= 1;
+            // per (row, slot): the slot's byte offset inside its row of a K-major
+            // SW128 tile -- row n = kBRows bw + r at n * 128 B, 16-byte unit
+            // (k / 4) ^ (n % 8) with n % 8 = r % 8 -- is the same in every chunk
+            // (k = col - 32 c changes k / 4 by multiples of 8), so it is formed
+            // once; packed with the slot's chunk (bits 16..) and the lo part
+            int32_t pk[kBRows];
+            float vlo[kBRows];
+#pragma unroll
+            for (int r = 0; r < kBRows; r++) {
+                const int32_t k = col[r];
+                pk[r] = k < 0 ? -1
+                              : (r * 128 + (((((uint32_t)k >> 2) ^ (uint32_t)r) & 7u) << 4) + ((k & 3) << 2)) |
+                                    ((k >> 5) << 16);
+                vlo[r] = tf32_lo(val[r]);
+            }
 #ifdef LF_TC_TRACE
             if (lane == 0) atomicAdd(&lf_tc_trace[blockIdx.x][16], (unsigned long long)(clock64() - tb0));
 #endif
@@ -524,16 +554,12 @@ __global__ void __launch_bounds__(kTcWarps * 32, 1) cell_spmm_tc_kernel(const Sp
                     *reinterpret_cast<float4 *>(tl + (u * 32 + lane) * 16) = make_float4(0.f, 0.f, 0.f, 0.f);
                 }
                 __syncwarp();
-                const int kb = kTcK * c;
 #pragma unroll
                 for (int r = 0; r < kBRows; r++) {
-                    // row n = kBRows bw + r of a K-major SW128 tile: n * 128 bytes,
-                    // 16-byte unit (k / 4) ^ (n % 8), n % 8 = r % 8
-                    const int k = col[r] - kb;  // col = -1 gives k < 0: no store
-                    const int o = r * 128 + ((((uint32_t)k >> 2) ^ (uint32_t)(r & 7)) << 4) + ((k & 3) << 2);
-                    if ((unsigned)k < (unsigned)kTcK) {
+                    if ((pk[r] >> 16) == c) {  // slot in this chunk (pk = -1: none)
+                        const int o = pk[r] & 0xffff;
                         *reinterpret_cast<float *>(th + o) = val[r];
-                        *reinterpret_cast<float *>(tl + o) = tf32_lo(val[r]);
+                        *reinterpret_cast<float *>(tl + o) = vlo[r];
                     }
                 }
                 asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // generic writes -> tensor core reads
@@ -554,8 +580,8 @@ __global__ void __launch_bounds__(kTcWarps * 32, 1) cell_spmm_tc_kernel(const Sp
             constexpr uint32_t idesc = (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(kTcN >> 3) << 17) |
                                        ((uint32_t)(128 >> 4) << 24);  // F32 accum, TF32 A/B, K-major B, N, M = 128
             uint32_t sa = 0, pha = 0, sv = 0, phv = 0, d = 0, phd = 0;
-            for (int64_t g = blockIdx.x; g < n_groups; g += gridDim.x) {
-                const TcGroup x = tc_group(a, g, bcur);
+            for (TcIter it(a); it.g < n_groups; it.next(a)) {
+                const TcGroup &x = it.x;
                 if (!x.mma) continue;
                 TC_WAIT(7, &sm.empty_d[d], phd ^ 1);
                 tc_fence_after();
@@ -567,11 +593,17 @@ __global__ void __launch_bounds__(kTcWarps * 32, 1) cell_spmm_tc_kernel(const Sp
                     const int nks = min(kTcK / 8, (x.span - kTcK * c + 7) / 8);
                     const uint64_t dh = sw128_desc(sm.vhi[sv]), dl = sw128_desc(sm.vlo[sv]);
                     const uint32_t a_raw = tmem + kColA + 64 * sa;
+#ifdef LF_TC_TRACE
+                    const long long tm0 = clock64();
+#endif
                     for (int ks = 0; ks < nks; ks++) {
                         tc_mma(dcol, a_raw + 8 * ks, dh + 2 * ks, idesc, (c | ks) != 0);
                         tc_mma(dcol, a_raw + 32 + 8 * ks, dh + 2 * ks, idesc, 1);
                         tc_mma(dcol, a_raw + 8 * ks, dl + 2 * ks, idesc, 1);
                     }
+#ifdef LF_TC_TRACE
+                    atomicAdd(&lf_tc_trace[blockIdx.x][19], (unsigned long long)(clock64() - tm0));
+#endif
                     tc_commit(&sm.empty_a[sa]);
                     tc_commit(&sm.empty_v[sv]);
                     if (++sa == kTcAStages) {
@@ -593,8 +625,8 @@ __global__ void __launch_bounds__(kTcWarps * 32, 1) cell_spmm_tc_kernel(const Sp
         // B window in chunks of 32 rows, into their rings =====
         uint32_t sb = 0, phb = 0, sc = 0, phc = 0;
         const bool packed = a.ldb == a.J;
-        for (int64_t g = blockIdx.x; g < n_groups; g += gridDim.x) {
-            const TcGroup x = tc_group(a, g, bcur);
+        for (TcIter it(a); it.g < n_groups; it.next(a)) {
+            const TcGroup &x = it.x;
             if (!x.mma) continue;
             {
                 const int64_t s0 = x.slot0 & ~int64_t(3);
@@ -722,7 +754,7 @@ cudaError_t launch_cell_spmm_tc(const SpmmArgs &a, cudaStream_t s) {
     const char *names[24] = {"ld:full_m", "ld:full_b", "ld:empty_a", "ep:full_d", "bu:full_c", "bu:empty_m",
                              "bu:empty_v", "mma:empty_d", "mma:full_a", "mma:full_v", "tma:empty_c", "tma:empty_b",
                              "T:loaders", "T:epilogue", "T:builders", "T:mma/tma", "bu:extract", "bu:chunks",
-                             "bu:tcgroup", "ep:stores", "ld:work", "x", "x", "x"};
+                             "bu:tcgroup", "mma:issue", "ld:work", "x", "x", "x"};
     fprintf(stderr, "tc trace (grid %d, mean cycles per CTA):", grid);
     for (int k = 0; k < 21; k++) {
         double sum = 0;
