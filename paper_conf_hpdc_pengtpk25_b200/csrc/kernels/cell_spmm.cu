@@ -132,6 +132,38 @@ template <> struct Vec<4> {
                      : "memory");
     }
 };
+// 8 floats per lane: one 256-bit load (ld.global.nc.v8.f32, sm_100) per B-row
+// slice, half the gather instructions of float4 for the same row bytes
+struct f8 {
+    float4 a, b;
+};
+template <> struct Vec<8> {
+    using T = f8;
+    static __device__ __forceinline__ T zero() { return {make_float4(0.f, 0.f, 0.f, 0.f), make_float4(0.f, 0.f, 0.f, 0.f)}; }
+    static __device__ __forceinline__ T load(const float *p) {
+        T v;
+        asm("ld.global.nc.v8.f32 {%0, %1, %2, %3, %4, %5, %6, %7}, [%8];"
+            : "=f"(v.a.x), "=f"(v.a.y), "=f"(v.a.z), "=f"(v.a.w), "=f"(v.b.x), "=f"(v.b.y), "=f"(v.b.z), "=f"(v.b.w)
+            : "l"(p));
+        return v;
+    }
+    static __device__ __forceinline__ void fma(T &acc, float a, const T &b) {
+        Vec<4>::fma(acc.a, a, b.a);
+        Vec<4>::fma(acc.b, a, b.b);
+    }
+    static __device__ __forceinline__ void add_xor(T &acc, int o) {
+        Vec<4>::add_xor(acc.a, o);
+        Vec<4>::add_xor(acc.b, o);
+    }
+    static __device__ __forceinline__ void store(float *p, const T &v, uint64_t pol) {
+        Vec<4>::store(p, v.a, pol);
+        Vec<4>::store(p + 4, v.b, pol);
+    }
+    static __device__ __forceinline__ void red(float *p, const T &v) {
+        Vec<4>::red(p, v.a);
+        Vec<4>::red(p + 4, v.b);
+    }
+};
 template <> struct Vec<1> {
     using T = float;
     static __device__ __forceinline__ T zero() { return 0.f; }
@@ -673,10 +705,12 @@ __device__ __forceinline__ void wide_loop_tiled(const SpmmArgs &a, const Cx &cx0
 // is register-allocated alone.  Epilogue: empty C rows are zeroed.
 // resident blocks per SM: wider J slices per lane (NV float4) need more
 // registers for the accumulators and the gathers in flight (no spills)
-constexpr int min_blocks(int NV) { return NV >= 4 ? 2 : NV == 2 ? 3 : kMinBlocks; }
+constexpr int min_blocks(int NV, int VEC = 4) {
+    return NV * VEC >= 16 ? 2 : NV * VEC == 8 ? 3 : kMinBlocks;
+}
 
 template <int VEC, int G, int NV, bool FULL>
-__global__ void __launch_bounds__(kWarpsPerBlock * 32, min_blocks(NV)) cell_spmm_kernel(const SpmmArgs a) {
+__global__ void __launch_bounds__(kWarpsPerBlock * 32, min_blocks(NV, VEC)) cell_spmm_kernel(const SpmmArgs a) {
     using Cx = Ctx<VEC, G, NV, FULL>;
     using L = Layout<VEC, G, NV>;
     __shared__ __align__(16) WarpStage stage_buf[kWarpsPerBlock];
@@ -703,7 +737,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, min_blocks(NV)) cell_spmm
     // share of the rows; done first, the write traffic overlaps the gathers
     // of the warps already streaming instead of forming a tail phase
     if (kZero && LF_ZERO_FIRST)
-        zero_rows_warp(a.row_mode, a.n_rows, a.C, a.ldc, a.J, VEC == 4, 1u << kRowEmpty,
+        zero_rows_warp(a.row_mode, a.n_rows, a.C, a.ldc, a.J, VEC >= 4, 1u << kRowEmpty,
                        (int64_t)blockIdx.x * kWarpsPerBlock + w, nw, lane, pol);
     if ((int)blockIdx.x < a.blocks_n) {
         narrow_loop(a, cx, st, lane, nw, pol);
@@ -719,7 +753,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, min_blocks(NV)) cell_spmm
     asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_work));
 #endif
     if (kZero && !LF_ZERO_FIRST)
-        zero_rows_warp(a.row_mode, a.n_rows, a.C, a.ldc, a.J, VEC == 4, 1u << kRowEmpty,
+        zero_rows_warp(a.row_mode, a.n_rows, a.C, a.ldc, a.J, VEC >= 4, 1u << kRowEmpty,
                        (int64_t)blockIdx.x * kWarpsPerBlock + w, (int64_t)gridDim.x * kWarpsPerBlock, lane, pol);
     // the last warp out resets the queue counters for the next launch that
     // uses this slot (every claim of every warp is ordered before its fence)
@@ -1336,6 +1370,10 @@ cudaError_t run_mma(const SpmmArgs &a, cudaStream_t s) {
     return cudaLaunchKernelEx(&cfg, fn, a);
 }
 
+bool vec8_ok(const float *B, int64_t ldb, const float *C, int64_t ldc, int J) {
+    return J % 8 == 0 && ldb % 8 == 0 && ldc % 8 == 0 && ((uintptr_t)B & 31) == 0 && ((uintptr_t)C & 31) == 0;
+}
+
 bool vec4_ok(const float *B, int64_t ldb, const float *C, int64_t ldc, int J) {
     return J % 4 == 0 && ldb % 4 == 0 && ldc % 4 == 0 && ((uintptr_t)B & 15) == 0 && ((uintptr_t)C & 15) == 0;
 }
@@ -1393,6 +1431,15 @@ cudaError_t launch_cell_spmm(const SpmmArgs &a, cudaStream_t s) {
     const bool tiled = v4 ? a.J > 512 : a.J > 128;
     cudaError_t e = zero_red_rows(a, tiled, s);
     if (e != cudaSuccess) return e;
+#ifndef LF_VEC8
+#define LF_VEC8 1  // 256-bit B-row gathers where J % 8 == 0 and B / C rows are 32-byte aligned
+#endif
+    // measured: c2 J = 128 0.603 -> 0.592 ms, c4 J = 256 6.01 -> 5.76 ms; J = 64 slower (0.363 -> 0.390)
+    if (LF_VEC8 && vec8_ok(a.B, a.ldb, a.C, a.ldc, a.J) && a.J > 64) {
+        if (a.J <= 128) return run_cell_j<8, 2, 1>(a, s);
+        if (a.J <= 256) return run_cell_j<8, 1, 1>(a, s);
+        return run_cell_j<8, 1, 2>(a, s);
+    }
     if (v4) {
         if (a.J <= 32) return run_cell_j<4, 4, 1>(a, s);
         if (a.J <= 64) return run_cell_j<4, 2, 1>(a, s);

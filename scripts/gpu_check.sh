@@ -5,9 +5,12 @@ mkdir -p gpurun_out
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv > gpurun_out/smi.txt 2>&1
 timeout 2400 python -m pytest tests -m gpu -x -q -p no:cacheprovider > gpurun_out/pytest_gpu.log 2>&1; echo "pytest rc=$?" >> gpurun_out/pytest_gpu.log
 timeout 900 python bench.py > gpurun_out/bench.json 2> gpurun_out/bench.err; echo "bench rc=$?" >> gpurun_out/bench.err
+timeout 900 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/bench_ref.json 2> gpurun_out/bench_ref.err
 timeout 900 python scripts/ncu_traffic.py > gpurun_out/traffic.log 2>&1
 cp profiles/traffic.json gpurun_out/traffic.json 2>/dev/null
+if [ "${SANITIZE:-1}" = "1" ]; then
 for tool in memcheck racecheck synccheck initcheck; do
-  timeout 1200 compute-sanitizer --tool $tool --target-processes all python scripts/sanitize_cases.py > gpurun_out/sanitize_$tool.log 2>&1
+  timeout 1500 compute-sanitizer --tool $tool --target-processes all python scripts/sanitize_cases.py > gpurun_out/sanitize_$tool.log 2>&1
   echo "rc=$?" >> gpurun_out/sanitize_$tool.log
 done
+fi

@@ -1,7 +1,7 @@
 """Small inputs through every kernel of liblf.so, for compute-sanitizer
 (memcheck / racecheck / synccheck / initcheck): configure (speculative and
 features-first paths), build (stats-sized and GPU-counted), the per-slot,
-grouped, tensor-core and CSR SpMM kernels, P > 1, folded rows, J tails.
+grouped, mma.sync, tcgen05 (windowed) and CSR SpMM kernels, P > 1, folded rows, J tails.
 Checks results against the oracle so a run that "passes" computed the right
 thing.   python scripts/sanitize_cases.py"""
 import os
@@ -26,17 +26,20 @@ cases = [(gen.config("c1_uniform1024", kind=gen.INT)[0], (32, 7)),
          (gen.rmat(10, 16, seed=1, kind=gen.INT), (64, 128)),
          (gen.banded(2048, 12, seed=2, kind=gen.INT), (64, 128)),
          (gen.arrowhead(2048, 4, seed=3, kind=gen.INT), (32,))]
+os.environ["LF_TC"] = "1"  # build the per-group windows of the tcgen05 path in every handle
 for A_h, Js in cases:
     A = lf.Csr.from_host(A_h)
     for J in Js:
         for P in (1, 3):
             params, stats = lf.configure(A, J, force_parts=P, force_format=1)
             for M in (lf.CellMatrix.build(A, params, stats), lf.CellMatrix.build(A, params)):
+                os.environ["LF_TC"] = "0"
                 check(M, A_h, J)
-                for env in ("LF_GROUPED", "LF_MMA"):
+                for env in ("LF_GROUPED", "LF_MMA", "LF_TC"):
                     os.environ[env] = "1"
                     check(M, A_h, J, env)
-                    del os.environ[env]
+                    os.environ[env] = "0"
+                os.environ["LF_TC"] = "1"
                 M.close()
         params, stats = lf.configure(A, J)  # predictor path
         M = lf.CellMatrix.build(A, params, stats)
