@@ -305,6 +305,10 @@ def main():
                     help="further workloads timed in the same run, name:J comma-separated ('none' to skip): each "
                          "gets its SpMM-only time, step time and roofline block")
     ap.add_argument("--shard-mode", default="nnz", choices=["nnz", "bytes"])
+    ap.add_argument("--exchange", default="nccl", choices=["nccl", "fused"],
+                    help="N > 1: C rows exchanged by NCCL point-to-point after the SpMM (nccl) or written by the "
+                         "SpMM kernels straight into every rank's symmetric-memory C over NVLink (fused, "
+                         "lf_spmm_ex destinations)")
     ap.add_argument("--streams", type=int, default=2,
                     help="steps in flight: consecutive steps alternate over this many CUDA streams, each with its "
                          "own C, so one step's host synchronisations (configure, build) overlap the previous "
@@ -367,10 +371,23 @@ def main():
     # steps in flight: lane l owns a stream and its own C (lane 0 reuses C_loc)
     n_lanes = max(1, args.streams)
     lanes = [torch.cuda.current_stream()] + [torch.cuda.Stream(dev) for _ in range(n_lanes - 1)]
-    lane_C = [(C_full, C_loc)]
-    for _ in range(n_lanes - 1):
-        Cf = torch.empty((A_h.n_rows, J), dtype=torch.float32, device=dev) if world > 1 else None
-        lane_C.append((Cf, Cf[lo:hi] if world > 1 else torch.empty((I_loc, J), dtype=torch.float32, device=dev)))
+    fused = world > 1 and args.exchange == "fused"
+    lane_sym = []
+    if fused:  # every lane: a symmetric-memory full C and the addresses of every rank's copy
+        lane_C = []
+        for _ in range(n_lanes):
+            sym = lfd.symmetric_C(A_h.n_rows, J, dev)
+            if sym is None:
+                raise SystemExit("bench.py: --exchange fused needs torch symmetric memory on this box")
+            lane_sym.append(sym)
+            lane_C.append((sym[0], sym[0][lo:hi]))
+        C_full, C_loc = lane_C[0]
+    else:
+        lane_C = [(C_full, C_loc)]
+        for _ in range(n_lanes - 1):
+            Cf = torch.empty((A_h.n_rows, J), dtype=torch.float32, device=dev) if world > 1 else None
+            lane_C.append((Cf, Cf[lo:hi] if world > 1 else torch.empty((I_loc, J), dtype=torch.float32,
+                                                                         device=dev)))
     h_C = torch.empty((I_loc, J), dtype=torch.float32).pin_memory()
     stream = torch.cuda.current_stream()
     kw = {}
@@ -391,9 +408,14 @@ def main():
             e1 = ev(); e1.record(st)
             M = lf.CellMatrix.build(Ain, params, stats, stream=st)
             e2 = ev(); e2.record(st)
-            M.spmm(d_B, out=Cl, stream=st)
+            if fused:  # the kernels write this rank's rows into every rank's C
+                M.spmm(d_B, stream=st, dst=lane_sym[lane][2], row_base=lo)
+            else:
+                M.spmm(d_B, out=Cl, stream=st)
             e3 = ev(); e3.record(st)
-            if world > 1:
+            if fused:
+                lane_sym[lane][1].barrier(channel=0)  # peers' rows landed before C is read
+            elif world > 1:
                 lfd.exchange_rows(Cf, bounds)  # NCCL ordered after this lane's stream
             e4 = ev(); e4.record(st)
         if record:
@@ -532,6 +554,8 @@ def main():
                    "cell_slots": info.get("cell_slots"),
                    "cell_rows": info.get("cell_rows"), "n_buckets": info.get("n_buckets"),
                    "parallelism": f"rows{world}", "shard_mode": args.shard_mode, "streams": n_lanes,
+                   "exchange": ("fused (SpMM writes every rank's symmetric C)" if fused else
+                                "nccl p2p after the SpMM") if world > 1 else "none",
                    "l2": "inputs larger than L2 (B, C, CELL each >126 MB); no flush"},
         "phases_ms": ph,
         "ms_per_step_serial": ms_serial if ms_serial is not None else ms,

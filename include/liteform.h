@@ -258,6 +258,35 @@ LF_API lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, co
 LF_API lf_status lf_spmm(const lf_cell *h, const float *B, int64_t ldb, int32_t J, float *C, int64_t ldc,
                   lf_stream_t s);
 
+/* Options of lf_spmm_ex: the FUSED ROW EXCHANGE of row-sharded multi-GPU SpMM
+ * (SURVEY 8(e), 8(f) NEXT-3).  With n_dst > 0 the kernels write every C row
+ * i of this handle's A straight from registers into each destination C,
+ * dst[d] + (row_base + i) * ldc -- the rank's own full C and its peers' C
+ * buffers mapped over NVLink (peer / symmetric memory) -- instead of C: the
+ * transfer overlaps the compute, and no separate all-gather follows.
+ *   n_dst     0 (plain lf_spmm) or 1..LF_MAX_DST
+ *   dst       (host) array of n_dst (device) pointers, each the base of a full
+ *             I_total x ldc C; read during the call (copied into the launch's
+ *             slot of the handle), may be freed when it returns
+ *   row_base  first row of this handle's rows in every destination
+ * The caller orders reads of a peer's rows after that peer's launch (e.g. a
+ * barrier); rows written with red.add (several CELL rows per C row) are
+ * pre-zeroed in every destination by the same launch. */
+#define LF_MAX_DST 8
+typedef struct lf_spmm_opts {
+    int32_t n_dst;
+    int32_t pad_;
+    float *const *dst;
+    int64_t row_base;
+} lf_spmm_opts;
+
+/* lf_spmm with options (opts may be NULL = lf_spmm).  C may be NULL when
+ * n_dst > 0.  Errors as lf_spmm, plus LF_ERR_INVALID_ARG (n_dst outside
+ * [0, LF_MAX_DST], NULL dst or destination, row_base < 0) and
+ * LF_ERR_UNSUPPORTED (n_dst > 0 on a handle built with use_cell = 0). */
+LF_API lf_status lf_spmm_ex(const lf_cell *h, const float *B, int64_t ldb, int32_t J, float *C, int64_t ldc,
+                            const lf_spmm_opts *opts, lf_stream_t s);
+
 /* Name of the SpMM kernel family lf_spmm runs for this handle at this J
  * with 16-byte aligned B / C and ldb = ldc = J (e.g. "cell_spmm_kernel",
  * "cell_spmm_grouped_kernel", "cell_spmm_tc_kernel", "csr_spmm_kernel";

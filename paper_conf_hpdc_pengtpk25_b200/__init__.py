@@ -136,13 +136,41 @@ class CellMatrix:
                                      ctypes.byref(_abi.torch_allocator()), _stream(stream), ctypes.byref(h)))
         return CellMatrix(h, A, params)
 
-    def spmm(self, B: torch.Tensor, out: torch.Tensor | None = None, stream=None) -> torch.Tensor:
-        """C = A . B (overwrites out).  B: [K, J] fp32 CUDA, row-major (row stride = ldb)."""
+    def spmm(self, B: torch.Tensor, out: torch.Tensor | None = None, stream=None, dst=None,
+             row_base: int = 0) -> torch.Tensor | None:
+        """C = A . B (overwrites out).  B: [K, J] fp32 CUDA, row-major (row stride = ldb).
+
+        dst: fused row exchange (lf_spmm_ex) -- a list of full-C destinations
+        (tensors [I_total, J] with unit column stride and a common row stride,
+        or raw device addresses); row i of this matrix is written to row
+        row_base + i of every destination straight from the kernel, and out is
+        not used.  Returns out (None with dst)."""
         if B.dtype != torch.float32 or not B.is_cuda or B.dim() != 2 or B.stride(1) != 1:
             raise TypeError("B must be a 2-D CUDA float32 tensor with unit column stride")
         if B.shape[0] != self.n_cols:
             raise ValueError(f"B has {B.shape[0]} rows, A has {self.n_cols} columns")
         J = B.shape[1]
+        if dst is not None:
+            ptrs, ldc = [], None
+            for t in dst:
+                if isinstance(t, torch.Tensor):
+                    if t.dtype != torch.float32 or t.dim() != 2 or t.stride(1) != 1 or t.shape[1] != J:
+                        raise ValueError("each destination must be [I_total, J] float32 with unit column stride")
+                    if t.shape[0] < row_base + self.n_rows:
+                        raise ValueError("destination has fewer rows than row_base + n_rows")
+                    if ldc is not None and t.stride(0) != ldc:
+                        raise ValueError("destinations must share one row stride")
+                    ldc = t.stride(0)
+                    ptrs.append(t.data_ptr())
+                else:
+                    ptrs.append(int(t))
+            ldc = max(ldc or J, J)
+            arr = (ctypes.c_void_p * len(ptrs))(*ptrs)
+            opts = _abi.LfSpmmOpts(len(ptrs), 0, ctypes.cast(arr, ctypes.POINTER(ctypes.c_void_p)), int(row_base))
+            self._J = J
+            _abi.check(lib.lf_spmm_ex(self._h, B.data_ptr(), max(B.stride(0), J), J, None, ldc, ctypes.byref(opts),
+                                      _stream(stream)))
+            return None
         if out is None:
             out = torch.empty((self.n_rows, J), dtype=torch.float32, device=B.device)
         if out.shape != (self.n_rows, J) or out.stride(1) != 1 or out.dtype != torch.float32:

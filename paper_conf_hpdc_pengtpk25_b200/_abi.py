@@ -78,6 +78,13 @@ class LfCellArrays(ctypes.Structure):
                 ("buckets", ctypes.POINTER(LfBucket)), ("params", LfCellParams)]
 
 
+LF_MAX_DST = 8
+
+
+class LfSpmmOpts(ctypes.Structure):
+    _fields_ = [("n_dst", _I32), ("pad_", _I32), ("dst", ctypes.POINTER(ctypes.c_void_p)), ("row_base", _I64)]
+
+
 # every symbol include/liteform.h declares, with its ctypes signature
 SIGNATURES = {
     "lf_cell_configure": (_I32, [ctypes.POINTER(LfCsr), _I32, ctypes.POINTER(LfConfigureOpts),
@@ -87,6 +94,7 @@ SIGNATURES = {
     "lf_spmm": (_I32, [_P, _P, _I64, _I32, _P, _I64, _P]),
     "lf_predict": (_I32, [ctypes.POINTER(ctypes.c_double), _I32, ctypes.POINTER(_I32), ctypes.POINTER(_I32)]),
     "lf_spmm_kernel_name": (ctypes.c_char_p, [_P, _I32]),
+    "lf_spmm_ex": (_I32, [_P, _P, _I64, _I32, _P, _I64, ctypes.POINTER(LfSpmmOpts), _P]),
     "lf_csr_spmm": (_I32, [ctypes.POINTER(LfCsr), _P, _I64, _I32, _P, _I64, _P]),
     "lf_cell_view": (_I32, [_P, ctypes.POINTER(LfCellArrays)]),
     "lf_cell_destroy": (_I32, [_P]),

@@ -215,6 +215,9 @@ struct Ctx {
     int j0;
     int g, li;  // lane group, lane in group
     uint64_t pol;
+    int nd = 0;                  // fused row exchange: destinations (0: C)
+    float *const *dp = nullptr;  // (device) destination bases
+    int64_t rb = 0;              // row offset of this matrix in every destination
 
     __device__ __forceinline__ int jcol(int m) const { return j0 + (m * L::LPR + li) * VEC; }
     __device__ __forceinline__ bool jok(int m) const { return FULL || jcol(m) < J; }
@@ -235,8 +238,7 @@ struct Ctx {
         for (int m = 0; m < NV; m++) b[m] = (jok(m) && real) ? V::load(r + jcol(m)) : V::zero();
     }
     // write one C row slice: plain store when this write is the row's only one
-    __device__ __forceinline__ void write(int32_t row, bool plain, const VT (&acc)[NV]) const {
-        float *p = C + (int64_t)row * ldc;
+    __device__ __forceinline__ void write_to(float *p, bool plain, const VT (&acc)[NV]) const {
 #pragma unroll
         for (int m = 0; m < NV; m++) {
             if (!jok(m)) continue;
@@ -246,6 +248,16 @@ struct Ctx {
             if (plain) V::store(p + jcol(m), acc[m], pol);
             else V::red(p + jcol(m), acc[m]);
         }
+    }
+    // write one C row slice (plain store when this write is the row's only
+    // one); with a fused row exchange, the same slice goes to every
+    // destination C (local and peers) straight from the registers
+    __device__ __forceinline__ void write(int32_t row, bool plain, const VT (&acc)[NV]) const {
+        if (nd == 0) {
+            write_to(C + (int64_t)row * ldc, plain, acc);
+            return;
+        }
+        for (int d = 0; d < nd; d++) write_to(ld_dst(dp, d) + (rb + row) * ldc, plain, acc);
     }
     __device__ __forceinline__ void zero(VT (&acc)[NV]) const {
 #pragma unroll
@@ -380,14 +392,16 @@ __device__ __forceinline__ void zero_row(float *row, int J, int lane, bool vec4,
 
 __device__ __forceinline__ void zero_rows_warp(const uint8_t *__restrict__ row_mode, int64_t n_rows, float *C,
                                                int64_t ldc, int J, bool vec4, unsigned mode_mask, int64_t wid,
-                                               int64_t nw, int lane, uint64_t pol) {
+                                               int64_t nw, int lane, uint64_t pol, int nd = 0,
+                                               float *const *dp = nullptr, int64_t rb = 0) {
     for (int64_t base = wid * 32; base < n_rows; base += nw * 32) {
         const int64_t i = base + lane;
         unsigned need = __ballot_sync(kFull, i < n_rows && ((mode_mask >> __ldg(row_mode + i)) & 1u));
         while (need) {
             const int src = __ffs(need) - 1;
             need &= need - 1;
-            zero_row(C + (base + src) * ldc, J, lane, vec4, pol);
+            if (nd == 0) zero_row(C + (base + src) * ldc, J, lane, vec4, pol);
+            for (int d = 0; d < nd; d++) zero_row(ld_dst(dp, d) + (rb + base + src) * ldc, J, lane, vec4, pol);
         }
     }
 }
@@ -718,7 +732,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, min_blocks(NV, VEC)) cell
     const int w = threadIdx.x >> 5;
     WarpStage &st = stage_buf[w];
     const uint64_t pol = policy_evict_first();
-    const Cx cx{a.B, a.ldb, a.C, a.ldc, a.J, 0, lane / L::LPR, lane % L::LPR, pol};
+    const Cx cx{a.B, a.ldb, a.C, a.ldc, a.J, 0, lane / L::LPR, lane % L::LPR, pol, a.n_dst, a.dst, a.row_base};
     const bool tiled = a.J > L::JT;
 #ifdef LF_TRACE
     {
@@ -738,7 +752,7 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, min_blocks(NV, VEC)) cell
     // of the warps already streaming instead of forming a tail phase
     if (kZero && LF_ZERO_FIRST)
         zero_rows_warp(a.row_mode, a.n_rows, a.C, a.ldc, a.J, VEC >= 4, 1u << kRowEmpty,
-                       (int64_t)blockIdx.x * kWarpsPerBlock + w, nw, lane, pol);
+                       (int64_t)blockIdx.x * kWarpsPerBlock + w, nw, lane, pol, a.n_dst, a.dst, a.row_base);
     if ((int)blockIdx.x < a.blocks_n) {
         narrow_loop(a, cx, st, lane, nw, pol);
         if (tiled) wide_loop_tiled(a, cx, st, lane, pol);
@@ -754,7 +768,8 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, min_blocks(NV, VEC)) cell
 #endif
     if (kZero && !LF_ZERO_FIRST)
         zero_rows_warp(a.row_mode, a.n_rows, a.C, a.ldc, a.J, VEC >= 4, 1u << kRowEmpty,
-                       (int64_t)blockIdx.x * kWarpsPerBlock + w, (int64_t)gridDim.x * kWarpsPerBlock, lane, pol);
+                       (int64_t)blockIdx.x * kWarpsPerBlock + w, (int64_t)gridDim.x * kWarpsPerBlock, lane, pol,
+                       a.n_dst, a.dst, a.row_base);
     // the last warp out resets the queue counters for the next launch that
     // uses this slot (every claim of every warp is ordered before its fence)
     if (lane == 0) {
@@ -809,13 +824,14 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32)
 }
 
 __global__ void zero_rows_kernel(const uint8_t *__restrict__ row_mode, int64_t n_rows, float *__restrict__ C,
-                                 int64_t ldc, int J, int vec4, unsigned mode_mask) {
+                                 int64_t ldc, int J, int vec4, unsigned mode_mask, int nd, float *const *dp,
+                                 int64_t rb) {
     asm volatile("griddepcontrol.launch_dependents;");
     const int lane = threadIdx.x & 31;
     const int64_t gwarp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
     const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
     zero_rows_warp(row_mode, n_rows, C, ldc, J, vec4 != 0, mode_mask, gwarp, nwarps, lane,
-                   policy_evict_first());
+                   policy_evict_first(), nd, dp, rb);
 }
 
 #ifndef LF_CARVEOUT
@@ -975,10 +991,10 @@ __global__ void __launch_bounds__(kWarpsPerBlock * 32, LF_GROUP_MIN_BLOCKS) cell
     for (int q = lane; q < kHT; q += 32) gs.key[q] = -1;
     __syncwarp();
     const uint64_t pol = policy_evict_first();
-    const Cx cx{a.B, a.ldb, a.C, a.ldc, a.J, 0, lane / L::LPR, lane % L::LPR, pol};
+    const Cx cx{a.B, a.ldb, a.C, a.ldc, a.J, 0, lane / L::LPR, lane % L::LPR, pol, a.n_dst, a.dst, a.row_base};
     const int64_t nw = (int64_t)gridDim.x * kWarpsPerBlock;
     zero_rows_warp(a.row_mode, a.n_rows, a.C, a.ldc, a.J, true, 1u << kRowEmpty,
-                   (int64_t)blockIdx.x * kWarpsPerBlock + w, nw, lane, pol);
+                   (int64_t)blockIdx.x * kWarpsPerBlock + w, nw, lane, pol, a.n_dst, a.dst, a.row_base);
     const unsigned lt = (1u << lane) - 1u;
     const int64_t n = a.n_groups;
     int bcur = 0;
@@ -1370,12 +1386,17 @@ cudaError_t run_mma(const SpmmArgs &a, cudaStream_t s) {
     return cudaLaunchKernelEx(&cfg, fn, a);
 }
 
-bool vec8_ok(const float *B, int64_t ldb, const float *C, int64_t ldc, int J) {
-    return J % 8 == 0 && ldb % 8 == 0 && ldc % 8 == 0 && ((uintptr_t)B & 31) == 0 && ((uintptr_t)C & 31) == 0;
+// c_bits: OR of every C base address the launch writes (C, or each fused-exchange destination)
+bool vec8_ok(const float *B, int64_t ldb, uintptr_t c_bits, int64_t ldc, int J) {
+    return J % 8 == 0 && ldb % 8 == 0 && ldc % 8 == 0 && ((uintptr_t)B & 31) == 0 && (c_bits & 31) == 0;
+}
+
+bool vec4_ok(const float *B, int64_t ldb, uintptr_t c_bits, int64_t ldc, int J) {
+    return J % 4 == 0 && ldb % 4 == 0 && ldc % 4 == 0 && ((uintptr_t)B & 15) == 0 && (c_bits & 15) == 0;
 }
 
 bool vec4_ok(const float *B, int64_t ldb, const float *C, int64_t ldc, int J) {
-    return J % 4 == 0 && ldb % 4 == 0 && ldc % 4 == 0 && ((uintptr_t)B & 15) == 0 && ((uintptr_t)C & 15) == 0;
+    return vec4_ok(B, ldb, (uintptr_t)C, ldc, J);
 }
 
 }  // namespace
@@ -1384,20 +1405,22 @@ bool vec4_ok(const float *B, int64_t ldb, const float *C, int64_t ldc, int J) {
 // kRowRun rows too when J needs several tiles (no run merging then)
 cudaError_t zero_red_rows(const SpmmArgs &a, bool tiled, cudaStream_t s) {
     if (a.n_rows == 0 || a.J == 0) return cudaSuccess;
-    const int vec4 = (a.J % 4 == 0 && a.ldc % 4 == 0 && ((uintptr_t)a.C & 15) == 0) ? 1 : 0;
+    const int vec4 = (a.J % 4 == 0 && a.ldc % 4 == 0 && (a.c_bits & 15) == 0) ? 1 : 0;
     const unsigned mask = (1u << kRowRed) | (tiled ? (1u << kRowRun) : 0u) | (LF_EPI_ZERO ? 0u : (1u << kRowEmpty));
     int64_t warps = (a.n_rows + 31) / 32;
     int grid = (int)std::max<int64_t>(1, std::min<int64_t>((warps + 7) / 8, (int64_t)sm_count() * 16));
-    zero_rows_kernel<<<grid, 256, 0, s>>>(a.row_mode, a.n_rows, a.C, a.ldc, a.J, vec4, mask);
+    zero_rows_kernel<<<grid, 256, 0, s>>>(a.row_mode, a.n_rows, a.C, a.ldc, a.J, vec4, mask, a.n_dst, a.dst,
+                                          a.row_base);
     return cudaGetLastError();
 }
 
 bool grouped_ok(const SpmmArgs &a) {
-    return a.grouped && a.nb_g > 0 && vec4_ok(a.B, a.ldb, a.C, a.ldc, a.J) && a.J <= 128;
+    return a.grouped && a.nb_g > 0 && vec4_ok(a.B, a.ldb, a.c_bits, a.ldc, a.J) && a.J <= 128;
 }
 
 bool mma_ok(const SpmmArgs &a) {
-    return a.mma && a.nb_g > 0 && vec4_ok(a.B, a.ldb, a.C, a.ldc, a.J) && a.J % 64 == 0 && a.J <= 128;
+    return a.mma && a.n_dst == 0 && a.nb_g > 0 && vec4_ok(a.B, a.ldb, a.c_bits, a.ldc, a.J) && a.J % 64 == 0 &&
+           a.J <= 128;
 }
 
 const char *cell_spmm_path(const SpmmArgs &a) {
@@ -1410,7 +1433,7 @@ const char *cell_spmm_path(const SpmmArgs &a) {
 
 cudaError_t launch_cell_spmm(const SpmmArgs &a, cudaStream_t s) {
     if (a.J == 0 || a.n_rows == 0) return cudaSuccess;
-    const bool v4 = vec4_ok(a.B, a.ldb, a.C, a.ldc, a.J);
+    const bool v4 = vec4_ok(a.B, a.ldb, a.c_bits, a.ldc, a.J);
     if (tc_ok(a)) {  // runs of folded rows are split across groups: red.add, pre-zeroed
         cudaError_t e = zero_red_rows(a, true, s);
         if (e != cudaSuccess) return e;
@@ -1435,7 +1458,7 @@ cudaError_t launch_cell_spmm(const SpmmArgs &a, cudaStream_t s) {
 #define LF_VEC8 1  // 256-bit B-row gathers where J % 8 == 0 and B / C rows are 32-byte aligned
 #endif
     // measured: c2 J = 128 0.603 -> 0.592 ms, c4 J = 256 6.01 -> 5.76 ms; J = 64 slower (0.363 -> 0.390)
-    if (LF_VEC8 && vec8_ok(a.B, a.ldb, a.C, a.ldc, a.J) && a.J > 64) {
+    if (LF_VEC8 && vec8_ok(a.B, a.ldb, a.c_bits, a.ldc, a.J) && a.J > 64) {
         if (a.J <= 128) return run_cell_j<8, 2, 1>(a, s);
         if (a.J <= 256) return run_cell_j<8, 1, 1>(a, s);
         return run_cell_j<8, 1, 2>(a, s);

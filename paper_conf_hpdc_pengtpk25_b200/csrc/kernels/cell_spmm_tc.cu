@@ -248,12 +248,14 @@ __device__ void zero_empty_rows(const SpmmArgs &a, int64_t wid, int64_t nw, int 
         while (need) {
             const int src = __ffs(need) - 1;
             need &= need - 1;
-            float *row = a.C + (base + src) * a.ldc;
-            for (int j = lane * 4; j < a.J; j += 128)
-                asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.f32 [%0], {%1, %1, %1, %1}, %2;" ::"l"(
-                                 row + j),
-                             "f"(0.f), "l"(pol)
-                             : "memory");
+            for (int d = 0; d < max(a.n_dst, 1); d++) {  // C, or every fused-exchange destination
+                float *row = (a.n_dst ? ld_dst(a.dst, d) + a.row_base * a.ldc : a.C) + (base + src) * a.ldc;
+                for (int j = lane * 4; j < a.J; j += 128)
+                    asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.f32 [%0], {%1, %1, %1, %1}, %2;" ::"l"(
+                                     row + j),
+                                 "f"(0.f), "l"(pol)
+                                 : "memory");
+            }
         }
     }
 }
@@ -279,8 +281,8 @@ __device__ void fallback_group(const SpmmArgs &a, const TcGroup &x, int bw, int 
                 acc.w = fmaf(v, b.w, acc.w);
             }
         }
-        if (j < a.J) {
-            float *p = a.C + (int64_t)tag_row(tag) * a.ldc + j;
+        for (int d = 0; d < max(a.n_dst, 1) && j < a.J; d++) {
+            float *p = (a.n_dst ? ld_dst(a.dst, d) + a.row_base * a.ldc : a.C) + (int64_t)tag_row(tag) * a.ldc + j;
             if (tag_whole(tag)) {
                 asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(p),
                              "f"(acc.x), "f"(acc.y), "f"(acc.z), "f"(acc.w), "l"(pol)
@@ -427,21 +429,25 @@ __global__ void __launch_bounds__(kTcWarps * 32, 1) cell_spmm_tc_kernel(const Sp
                 const int32_t tg = tags[nb];
                 const bool whole = tg < 0 || tag_whole(tg);
                 const long long roff = tg >= 0 ? (long long)tag_row(tg) * a.ldc : -1;
-                if (__all_sync(kFull, whole)) {
+                // C, or (fused row exchange) each destination C in turn
+                for (int dd = 0; dd < max(a.n_dst, 1); dd++) {
+                    float *const cb = (a.n_dst ? ld_dst(a.dst, dd) + a.row_base * a.ldc : a.C) + j;
+                    if (__all_sync(kFull, whole)) {
 #pragma unroll
-                    for (int i = 0; i < 32; i++) {
-                        const long long ro = __shfl_sync(kFull, roff, i);
-                        if (ro >= 0 && jok) __stcs(a.C + ro + j, __uint_as_float(v[i]));
-                    }
-                } else {
-                    grid_dep_wait();
+                        for (int i = 0; i < 32; i++) {
+                            const long long ro = __shfl_sync(kFull, roff, i);
+                            if (ro >= 0 && jok) __stcs(cb + ro, __uint_as_float(v[i]));
+                        }
+                    } else {
+                        grid_dep_wait();
 #pragma unroll
-                    for (int i = 0; i < 32; i++) {
-                        const long long ro = __shfl_sync(kFull, roff, i);
-                        const bool wh = __shfl_sync(kFull, whole, i);
-                        if (ro >= 0 && jok) {
-                            if (wh) __stcs(a.C + ro + j, __uint_as_float(v[i]));
-                            else atomicAdd(a.C + ro + j, __uint_as_float(v[i]));
+                        for (int i = 0; i < 32; i++) {
+                            const long long ro = __shfl_sync(kFull, roff, i);
+                            const bool wh = __shfl_sync(kFull, whole, i);
+                            if (ro >= 0 && jok) {
+                                if (wh) __stcs(cb + ro, __uint_as_float(v[i]));
+                                else atomicAdd(cb + ro, __uint_as_float(v[i]));
+                            }
                         }
                     }
                 }
@@ -720,7 +726,7 @@ cudaError_t launch_tc_windows(const BucketDev *bk_t, int nb_t, int64_t n_groups,
 
 bool tc_ok(const SpmmArgs &a) {
     return a.tc && a.nb_t > 0 && a.tc_win && a.J >= 32 && a.J <= 128 && a.J % 4 == 0 && a.ldb % 4 == 0 &&
-           a.ldc % 4 == 0 && ((uintptr_t)a.B & 15) == 0 && ((uintptr_t)a.C & 15) == 0;
+           a.ldc % 4 == 0 && ((uintptr_t)a.B & 15) == 0 && (a.c_bits & 15) == 0;
 }
 
 cudaError_t launch_cell_spmm_tc(const SpmmArgs &a, cudaStream_t s) {

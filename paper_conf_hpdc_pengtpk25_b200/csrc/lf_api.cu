@@ -171,7 +171,8 @@ lf::SpmmArgs spmm_args(const lf_cell *h, const float *B, int64_t ldb, int32_t J,
                    h->row_tag, B, ldb, C, ldc, J,
                    h->d_buckets + nb + h->nb_n + h->nb_w, h->nb_g, h->grouped, h->n_groups,
                    h->d_buckets + nb + h->nb_n + h->nb_w + h->nb_g, h->mma, h->n_groups_m,
-                   h->d_buckets + nb + h->nb_n + h->nb_w + 2 * h->nb_g, h->nb_g, h->tc, h->n_groups_t, h->tc_win};
+                   h->d_buckets + nb + h->nb_n + h->nb_w + 2 * h->nb_g, h->nb_g, h->tc, h->n_groups_t, h->tc_win,
+                   0, nullptr, 0, (uintptr_t)C};
     if (const char *g = std::getenv("LF_GROUPED")) a.grouped = g[0] == '1';
     if (const char *g = std::getenv("LF_TC")) a.tc = g[0] == '1';
     if (const char *g = std::getenv("LF_MMA")) a.mma = g[0] == '1';
@@ -589,7 +590,8 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
     const bool want_tc = h->nb_g > 0 && h->n_groups_t > 0 &&
                          (tc_env ? tc_env[0] == '1' : (stats ? stats->spmm_tc != 0 : true));
     const size_t b_tw = want_tc ? up((size_t)h->n_groups_t * sizeof(int2)) : 0;
-    h->pool_bytes = b_bk + b_ko + b_ri + b_rt + b_ci + b_va + b_rb + b_ct + b_rm + b_tw;
+    const size_t b_dr = up((size_t)kCtrSlots * lf::kMaxDst * sizeof(float *));
+    h->pool_bytes = b_bk + b_ko + b_ri + b_rt + b_ci + b_va + b_rb + b_ct + b_rm + b_tw + b_dr;
     h->pool = mem.get(h->pool_bytes);
     if (!h->pool) return bail(fail(LF_ERR_NO_MEMORY, "CELL arrays allocation failed"));
     char *q = static_cast<char *>(h->pool);
@@ -604,6 +606,7 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
     h->ctr_ring = reinterpret_cast<unsigned long long *>(q + b_ri + b_rt + b_ci + b_va + b_rb);
     h->row_mode = reinterpret_cast<uint8_t *>(q + b_ri + b_rt + b_ci + b_va + b_rb + b_ct);
     h->tc_win = b_tw ? reinterpret_cast<int2 *>(q + b_ri + b_rt + b_ci + b_va + b_rb + b_ct + b_rm) : nullptr;
+    h->dst_ring = reinterpret_cast<float **>(q + b_ri + b_rt + b_ci + b_va + b_rb + b_ct + b_rm + b_tw);
     {
         std::vector<char> head(b_bk + b_ko, 0);
         if (!h->h_buckets.empty())
@@ -641,20 +644,43 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
 
 lf_status lf_spmm(const lf_cell *h, const float *B, int64_t ldb, int32_t J, float *C, int64_t ldc,
                   lf_stream_t stream) {
+    return lf_spmm_ex(h, B, ldb, J, C, ldc, nullptr, stream);
+}
+
+lf_status lf_spmm_ex(const lf_cell *h, const float *B, int64_t ldb, int32_t J, float *C, int64_t ldc,
+                     const lf_spmm_opts *opts, lf_stream_t stream) {
     g_detail.clear();
     if (!h) return fail(LF_ERR_INVALID_ARG, "handle is NULL");
     if (J < 0 || ldb < J || ldc < J || ldb < 0 || ldc < 0) return fail(LF_ERR_INVALID_ARG, "need 0 <= J <= ldb, ldc");
+    const int n_dst = opts ? opts->n_dst : 0;
+    if (n_dst < 0 || n_dst > LF_MAX_DST) return fail(LF_ERR_INVALID_ARG, "n_dst outside [0, LF_MAX_DST]");
+    if (n_dst > 0) {
+        if (!opts->dst) return fail(LF_ERR_INVALID_ARG, "dst is NULL");
+        if (opts->row_base < 0) return fail(LF_ERR_INVALID_ARG, "row_base < 0");
+        for (int d = 0; d < n_dst; d++)
+            if (!opts->dst[d]) return fail(LF_ERR_INVALID_ARG, "a destination pointer is NULL");
+    }
     if (J == 0 || h->n_rows == 0) return LF_OK;
-    if (!C) return fail(LF_ERR_INVALID_ARG, "C is NULL");
+    if (!C && n_dst == 0) return fail(LF_ERR_INVALID_ARG, "C is NULL");
     if (!B && h->n_cols > 0) return fail(LF_ERR_INVALID_ARG, "B is NULL");
     cudaStream_t s = (cudaStream_t)stream;
     if (h->params.use_cell == 0) {
+        if (n_dst > 0) return fail(LF_ERR_UNSUPPORTED, "fused row exchange needs a CELL handle (use_cell = 1)");
         LF_CUDA(lf::launch_csr_spmm(h->csr, B, ldb, J, C, ldc, s));
         return LF_OK;
     }
     lf::SpmmArgs a = spmm_args(h, B, ldb, J, C, ldc);
     const uint32_t k = h->launch_seq.fetch_add(1, std::memory_order_relaxed) % kCtrSlots;
     a.ctr = h->ctr_ring + 4 * k;
+    if (n_dst > 0) {  // the destinations travel in the launch's own slot of the handle's ring
+        a.n_dst = n_dst;
+        a.dst = h->dst_ring + (size_t)k * lf::kMaxDst;
+        a.row_base = opts->row_base;
+        a.c_bits = 0;
+        for (int d = 0; d < n_dst; d++) a.c_bits |= (uintptr_t)opts->dst[d];
+        LF_CUDA(cudaMemcpyAsync(h->dst_ring + (size_t)k * lf::kMaxDst, opts->dst, (size_t)n_dst * sizeof(float *),
+                                cudaMemcpyHostToDevice, s));
+    }
     std::lock_guard<std::mutex> g(h->mu);
     if (s == h->stream && !h->multi) {  // the common case: one stream, launches ordered by it
         LF_CUDA(lf::launch_cell_spmm(a, s));

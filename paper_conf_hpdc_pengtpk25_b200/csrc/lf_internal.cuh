@@ -178,7 +178,18 @@ struct SpmmArgs {
     int tc;
     int64_t n_groups_t;
     const int2 *tc_win;
+    // fused row exchange (lf_spmm_ex): n_dst > 0 writes C row i to every
+    // dst[d] + (row_base + i) * ldc instead of C (peer C buffers over NVLink)
+    int n_dst;
+    float *const *dst;  // (device) [n_dst]
+    int64_t row_base;
+    uintptr_t c_bits;   // OR of the C / destination base addresses (alignment checks)
 };
+constexpr int kMaxDst = 8;
+// destination base d of a fused row exchange (read-only path)
+__device__ __forceinline__ float *ld_dst(float *const *dst, int d) {
+    return reinterpret_cast<float *>(__ldg(reinterpret_cast<const unsigned long long *>(dst) + d));
+}
 cudaError_t launch_cell_spmm(const SpmmArgs &a, cudaStream_t s);  // pre-zeroes kRowRed rows itself
 // name of the kernel launch_cell_spmm runs for these arguments
 const char *cell_spmm_path(const SpmmArgs &a);
@@ -237,6 +248,7 @@ struct lf_cell {
     mutable bool multi = false;
     mutable std::vector<std::pair<cudaStream_t, cudaEvent_t>> ext;
     mutable cudaEvent_t slot_ev[kCtrSlots] = {};
+    float **dst_ring = nullptr;  // [kCtrSlots][lf::kMaxDst] destination bases of lf_spmm_ex, per counter slot
     mutable cudaStream_t slot_stream[kCtrSlots] = {};
     mutable bool slot_recorded[kCtrSlots] = {};
 };

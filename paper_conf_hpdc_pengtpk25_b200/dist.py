@@ -115,6 +115,46 @@ def broadcast_B(B: torch.Tensor, src: int = 0, group=None) -> torch.Tensor:
     return B
 
 
+def symmetric_C(n_rows: int, J: int, device, group=None):
+    """A full [n_rows, J] C on every rank in symmetric memory (peer-mapped
+    over NVLink) and the device addresses of every rank's copy, rank order:
+    the destinations of the fused row exchange.  None where the process group
+    or device cannot provide symmetric memory."""
+    try:
+        import torch.distributed._symmetric_memory as symm
+        C = symm.empty((n_rows, J), dtype=torch.float32, device=device)
+        h = symm.rendezvous(C, group if group is not None else dist.group.WORLD)
+        return C, h, [int(p) for p in h.buffer_ptrs]
+    except Exception:  # pragma: no cover - depends on the box
+        return None
+
+
+def spmm_rowsharded_fused(A_full, B: torch.Tensor, J: int, group=None, mode: str = "nnz", **configure_kw):
+    """C = A . B with A's rows sharded and the C rows exchanged INSIDE the SpMM
+    (SURVEY 8(f) NEXT-3): every rank's kernels write their C rows straight into
+    every rank's symmetric-memory C (lf_spmm_ex destinations = all peers'
+    buffers over NVLink), so no all-gather follows the compute; a barrier over
+    the symmetric-memory signal pads orders the reads.  Returns (C, bounds);
+    falls back to spmm_rowsharded when symmetric memory is unavailable."""
+    from . import CellMatrix, Csr, configure
+    rank, world = dist.get_rank(group), dist.get_world_size(group)
+    sym = symmetric_C(A_full.n_rows, B.shape[1], B.device, group)
+    if sym is None:
+        return spmm_rowsharded(A_full, B, J, group, mode, True, **configure_kw)
+    C, h, ptrs = sym
+    rp_host = A_full.row_ptr.cpu().numpy()
+    bounds = shard_bounds(rp_host, world, J, mode)
+    lo, hi = int(bounds[rank]), int(bounds[rank + 1])
+    shard = Csr(A_full.row_ptr[lo:hi + 1], A_full.col_ind, A_full.val, A_full.n_cols,
+                int(rp_host[hi] - rp_host[lo]))
+    params, stats = configure(shard, J, force_format=1, **configure_kw)
+    M = CellMatrix.build(shard, params, stats)
+    M.spmm(B, dst=ptrs, row_base=lo)
+    if world > 1:
+        h.barrier(channel=0)
+    return C, bounds
+
+
 def spmm_rowsharded(A_full, B: torch.Tensor, J: int, group=None, mode: str = "nnz", gather: bool = True,
                     **configure_kw):
     """C = A . B with A's rows sharded over the group.  A_full is this rank's
