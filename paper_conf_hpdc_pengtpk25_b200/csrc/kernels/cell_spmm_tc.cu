@@ -210,11 +210,11 @@ __device__ __forceinline__ TcGroup tc_group(const SpmmArgs &a, int64_t g, int &b
     x.nr = (int)min((int64_t)kTcN, __ldg(&bk->n_rows_pad) - r0);
     x.row0 = __ldg(&bk->row_off) + r0;
     x.slot0 = __ldg(&bk->slot_off) + (r0 << x.t);
-    const int2 w = __ldg(a.tc_win + g);
+    const int2 w = __ldg(a.tc_win + g);  // {lo, span}; span 0: no real slot
     x.lo = w.x;
     x.span = w.y;
-    x.nch = (w.y + kTcK - 1) / kTcK;
-    x.mma = w.y > 0 && x.nch <= kTcMaxChunks;
+    x.nch = (x.span + kTcK - 1) / kTcK;
+    x.mma = x.span > 0 && x.nch <= kTcMaxChunks;
     return x;
 }
 
@@ -679,37 +679,51 @@ __global__ void __launch_bounds__(kTcWarps * 32, 1) cell_spmm_tc_kernel(const Sp
 }
 
 // Per group of kTcN CELL rows: window = [min first real column, max last real
-// column] over its rows (columns are sorted within a CELL row, R6).  One warp
-// per group, lane r reading rows r, r + 32, ... (2 loads per row).
-__global__ void tc_window_kernel(const BucketDev *__restrict__ bk, int nb, int64_t n_groups,
-                                 const int32_t *__restrict__ col, const int32_t *__restrict__ src_cnt,
-                                 int2 *__restrict__ win) {
-    const int lane = threadIdx.x & 31;
-    const int64_t nw = ((int64_t)gridDim.x * blockDim.x) >> 5;
-    int bcur = 0;
-    for (int64_t g = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; g < n_groups; g += nw) {
-        int lo_b = 0, hi_b = nb - 1;  // bucket of group g (binary search: grid-stride order)
+// column] over its rows (columns are sorted within a CELL row, R6).  One
+// 128-thread block per group, thread n reading row n (its real-slot count and
+// two columns: every load of the group in flight at once), block min / max.
+// (Folding this reduction into slot_fill with atomics measured slower: 181 ->
+// 253-371 us on c3b, vs 40 us for this kernel.)
+__global__ void __launch_bounds__(kTcN) tc_window_kernel(const BucketDev *__restrict__ bk, int nb, int64_t n_groups,
+                                                         const int32_t *__restrict__ col,
+                                                         const int32_t *__restrict__ src_cnt,
+                                                         int2 *__restrict__ win) {
+    __shared__ int smn[kTcN / 32], smx[kTcN / 32];
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+    for (int64_t g = blockIdx.x; g < n_groups; g += gridDim.x) {
+        int lo_b = 0, hi_b = nb - 1;  // bucket of group g
         while (lo_b < hi_b) {
             const int m = (lo_b + hi_b + 1) >> 1;
-            if (bk[m].task_off <= g) lo_b = m;
+            if (__ldg(&bk[m].task_off) <= g) lo_b = m;
             else hi_b = m - 1;
         }
-        bcur = lo_b;
-        const BucketDev b = bk[bcur];
-        const int64_t r0 = (g - b.task_off) * kTcN;
-        const int nr = (int)min((int64_t)kTcN, b.n_rows_pad - r0);
+        const BucketDev &b = bk[lo_b];
+        const int64_t r0 = (g - __ldg(&b.task_off)) * kTcN;
+        const int n = threadIdx.x;
         int mn = INT32_MAX, mx = -1;
-        for (int n = lane; n < nr; n += 32) {
-            const int cnt = src_cnt[b.row_off + r0 + n];
+        if (r0 + n < __ldg(&b.n_rows_pad)) {
+            const int cnt = __ldg(src_cnt + __ldg(&b.row_off) + r0 + n);
             if (cnt > 0) {
-                const int64_t s = b.slot_off + ((r0 + n) << b.t);
-                mn = min(mn, col[s]);
-                mx = max(mx, col[s + cnt - 1]);
+                const int64_t s = __ldg(&b.slot_off) + ((r0 + n) << __ldg(&b.t));
+                mn = __ldg(col + s);
+                mx = __ldg(col + s + cnt - 1);
             }
         }
         mn = __reduce_min_sync(kFull, mn);
         mx = __reduce_max_sync(kFull, mx);
-        if (lane == 0) win[g] = mx < 0 ? make_int2(0, 0) : make_int2(mn, mx - mn + 1);
+        if (lane == 0) {
+            smn[w] = mn;
+            smx[w] = mx;
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            for (int q = 1; q < kTcN / 32; q++) {
+                mn = min(mn, smn[q]);
+                mx = max(mx, smx[q]);
+            }
+            win[g] = mx < 0 ? make_int2(0, 0) : make_int2(mn, mx - mn + 1);
+        }
+        __syncthreads();
     }
 }
 
@@ -718,9 +732,8 @@ __global__ void tc_window_kernel(const BucketDev *__restrict__ bk, int nb, int64
 cudaError_t launch_tc_windows(const BucketDev *bk_t, int nb_t, int64_t n_groups, const int32_t *col,
                               const int32_t *src_cnt, int2 *win, cudaStream_t s) {
     if (n_groups == 0) return cudaSuccess;
-    const int64_t want = (n_groups * 32 + 255) / 256;
-    const int grid = (int)std::max<int64_t>(1, std::min<int64_t>(want, (int64_t)sm_count() * 8));
-    tc_window_kernel<<<grid, 256, 0, s>>>(bk_t, nb_t, n_groups, col, src_cnt, win);
+    const int grid = (int)std::min<int64_t>(n_groups, (int64_t)sm_count() * 64);
+    tc_window_kernel<<<grid, kTcN, 0, s>>>(bk_t, nb_t, n_groups, col, src_cnt, win);
     return cudaGetLastError();
 }
 

@@ -556,7 +556,7 @@ cudaError_t launch_features(const lf_csr &A, StatsDev *d_stats, cudaStream_t s) 
 }
 
 cudaError_t launch_stats(const lf_csr &A, int P, StatsDev *d_stats, uint32_t *d_colmask, uint8_t *d_t0seg,
-                         cudaStream_t s) {
+                         cudaStream_t s, bool sample) {
     const int64_t S = A.n_cols > 0 ? (A.n_cols + P - 1) / P : 1;
     const size_t hist = 2 * (size_t)P * kMaxT * sizeof(unsigned long long);
     if (A.n_rows > 0) {
@@ -576,7 +576,7 @@ cudaError_t launch_stats(const lf_csr &A, int P, StatsDev *d_stats, uint32_t *d_
                                                                     tile_row, tile_pos, tiles, d_colmask,
                                                                     mask_slots(A.n_cols) - 1);
     }
-    if (A.n_rows >= kGroupRows && A.nnz > 0)
+    if (sample && A.n_rows >= kGroupRows && A.nnz > 0)
         group_sample_kernel<<<kGroupSamples / 8, 256, 0, s>>>(A.row_ptr, A.col_ind, A.n_rows, d_stats);
     if (A.n_cols > 0) {
         const int64_t want = ((int64_t)mask_slots(A.n_cols) + kThreads - 1) / kThreads;

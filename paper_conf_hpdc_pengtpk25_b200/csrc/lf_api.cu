@@ -222,7 +222,11 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
     if (!h_st) LF_CUDA(cudaMallocHost(&h_st, sizeof(lf::StatsDev)));
     // GPU statistics for P partitions (one scratch allocation: stats, column
     // masks, per-segment t0 + mark tiles), copied back with one sync
+    bool sampled = false;  // group / window samples already in h_st (they do not depend on P)
     auto run_stats = [&](int P) -> lf_status {
+        const unsigned long long keep[5] = {h_st->grp_union, h_st->grp_nnz, h_st->win_span, h_st->win_cnt,
+                                            h_st->win_over};
+        const bool sample = !sampled;
         const size_t st_bytes = lf::stats_bytes(P);
         const size_t words = A->n_cols > 0 ? lf::mask_slots(A->n_cols) : 0;
         const size_t b_st = (st_bytes + 255) & ~size_t(255), b_mask = (words * 4 + 255) & ~size_t(255);
@@ -235,10 +239,18 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
         // stats and masks are adjacent: one memset zeroes both
         LF_CUDA(cudaMemsetAsync(d, 0, b_st + b_mask, s));
         LF_CUDA(cudaMemsetAsync(&d_st->len_min, 0xFF, sizeof(unsigned long long), s));
-        LF_CUDA(lf::launch_stats(*A, P, d_st, d_mask, d_t0, s));
+        LF_CUDA(lf::launch_stats(*A, P, d_st, d_mask, d_t0, s, sample));
         LF_CUDA(cudaMemcpyAsync(h_st, d_st, st_bytes, cudaMemcpyDeviceToHost, s));
         LF_CUDA(cudaFreeAsync(d, s));
         LF_CUDA(cudaStreamSynchronize(s));
+        if (!sample) {
+            h_st->grp_union = keep[0];
+            h_st->grp_nnz = keep[1];
+            h_st->win_span = keep[2];
+            h_st->win_cnt = keep[3];
+            h_st->win_over = keep[4];
+        }
+        sampled = true;
         return LF_OK;
     };
     // predictor (sections 5.1-5.2): it needs the Table 2 row-length features
@@ -267,6 +279,7 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
             LF_CUDA(cudaMemcpyAsync(h_st, d_f, fb, cudaMemcpyDeviceToHost, s));
             LF_CUDA(cudaFreeAsync(d_f, s));
             LF_CUDA(cudaStreamSynchronize(s));
+            sampled = A->n_rows >= lf::kGroupRows && A->nnz > 0;
         }
         double f[8];
         table2_features(*A, J, *h_st, f);
@@ -638,6 +651,7 @@ lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_
                                        h->col_ind, bs.src_cnt, h->tc_win, s),
                  "tc_windows")))
         return bail(st);
+
     *out = h;
     return LF_OK;
 }

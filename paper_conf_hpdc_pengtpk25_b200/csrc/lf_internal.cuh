@@ -82,8 +82,10 @@ inline size_t stats_bytes(int P) { return offsetof(StatsDev, part) + (size_t)P *
 uint32_t mask_slots(int64_t n_cols);  // words of the column-mask array (power of two >= K)
 size_t stats_scratch_bytes(int64_t n_rows, int64_t nnz, int P);  // t0 per segment + tile -> row map
 cudaError_t launch_features(const lf_csr &A, StatsDev *d_stats, cudaStream_t s);  // len_* only
+// sample = false: the group / window samples (independent of P) are already
+// known from an earlier pass over the same A and are not recomputed
 cudaError_t launch_stats(const lf_csr &A, int P, StatsDev *d_stats, uint32_t *d_colmask, uint8_t *d_t0seg,
-                         cudaStream_t s);
+                         cudaStream_t s, bool sample = true);
 
 struct BuildScratch {
     int32_t *seg_rel;       // [I*(P-1)] segment starts relative to the row start (P > 1)
@@ -194,11 +196,13 @@ cudaError_t launch_cell_spmm(const SpmmArgs &a, cudaStream_t s);  // pre-zeroes 
 // name of the kernel launch_cell_spmm runs for these arguments
 const char *cell_spmm_path(const SpmmArgs &a);
 // tcgen05 windowed path (cell_spmm_tc.cu)
-constexpr int kTcGroupRows = 128;
+constexpr int kTcGroupLog2 = 7;
+constexpr int kTcGroupRows = 1 << kTcGroupLog2;
 bool tc_ok(const SpmmArgs &a);
 cudaError_t launch_cell_spmm_tc(const SpmmArgs &a, cudaStream_t s);
 cudaError_t launch_tc_windows(const BucketDev *bk_t, int nb_t, int64_t n_groups, const int32_t *col,
                               const int32_t *src_cnt, int2 *win, cudaStream_t s);
+
 cudaError_t launch_csr_spmm(const lf_csr &A, const float *B, int64_t ldb, int J, float *C, int64_t ldc,
                             cudaStream_t s);
 cudaError_t launch_validate(const lf_csr &A, int *d_flag, cudaStream_t s);
