@@ -208,3 +208,32 @@ def test_tc_full_c3b(lf, monkeypatch, J):
     Mi = lf.CellMatrix.build(lf.Csr.from_host(Ai_h), params, stats)
     Ci = Mi.spmm(torch.from_numpy(Bi_h).cuda()).cpu().numpy().astype(np.float64)
     assert np.array_equal(Ci[rows], oracle.spmm_csr(Ai_h, Bi_h, rows)[0])
+
+
+def test_tc_edge_cases(lf, tc):
+    """No entries (C exactly +0.0), fewer rows than a group, a single column,
+    empty rows between real ones, J just above the 32 minimum; and J = 256 /
+    J = 16, which the windowed path does not take (per-slot / grouped path
+    instead, same result)."""
+    A_h = gen.CSR(7, 5, np.zeros(8, np.int64), np.zeros(0, np.int32), np.zeros(0, np.float32))
+    M = lf.CellMatrix.build(lf.Csr.from_host(A_h), lf.make_params(1, 2))
+    C = M.spmm(torch.full((5, 64), 3.0, device="cuda"), out=torch.full((7, 64), float("nan"), device="cuda"))
+    assert torch.equal(C, torch.zeros(7, 64, device="cuda"))
+    for I, K, J in ((1, 1, 32), (3, 1, 36), (130, 40, 64), (129, 300, 128), (5, 2, 16), (200, 200, 256)):
+        A_h = gen.random_small(I, K, 30, I + K, dup=True, zeros=True, kind=gen.INT)
+        B_h = gen.dense(K, J, 3, gen.INT, -15, 15)
+        C, M = run(lf, A_h, B_h, 1, 5)
+        assert np.array_equal(C, oracle.spmm_csr(A_h, B_h)[0]), (I, K, J)
+        want_tc = 32 <= J <= 128
+        assert (M.path(J) == "cell_spmm_tc_kernel") == want_tc, (J, M.path(J))
+    # rows with no entries interleaved with banded rows
+    A_b = gen.banded(1000, 12, seed=12, kind=gen.INT, lo=-3, hi=3)
+    keep = np.arange(1000) % 3 != 1
+    l = np.diff(A_b.row_ptr) * keep
+    rp = np.concatenate([[0], np.cumsum(l)]).astype(np.int64)
+    idx = np.concatenate([np.arange(A_b.row_ptr[i], A_b.row_ptr[i + 1]) for i in range(1000) if keep[i]])
+    A_h = gen.CSR(1000, 1000, rp, A_b.col_ind[idx], A_b.val[idx])
+    B_h = gen.dense(1000, 128, 4, gen.INT, -15, 15)
+    C, M = run(lf, A_h, B_h, 1, 5)
+    assert M.path(128) == "cell_spmm_tc_kernel"
+    assert np.array_equal(C, oracle.spmm_csr(A_h, B_h)[0])
