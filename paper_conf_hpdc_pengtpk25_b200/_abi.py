@@ -110,6 +110,8 @@ def load(path: str = LIB_PATH) -> ctypes.CDLL:
                           "(there is no CPU fallback)")
     L = ctypes.CDLL(path)
     for name, (res, args) in SIGNATURES.items():
+        if os.environ.get("LF_LIB") and not hasattr(L, name):
+            continue  # an experiment / comparison build of another revision (LF_LIB) may predate a call
         f = getattr(L, name)
         f.restype = res
         f.argtypes = args
