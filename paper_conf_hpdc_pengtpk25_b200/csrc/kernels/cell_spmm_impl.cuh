@@ -155,6 +155,11 @@ template <> struct Vec<8> {
             : "l"(p));
         return v;
     }
+                : "=f"(v.a.x), "=f"(v.a.y), "=f"(v.a.z), "=f"(v.a.w), "=f"(v.b.x), "=f"(v.b.y), "=f"(v.b.z), "=f"(v.b.w)
+                : "l"(p));
+        return v;
+    }
+#endif
     static __device__ __forceinline__ void fma(T &acc, float a, const T &b) {
         Vec<4>::fma(acc.a, a, b.a);
         Vec<4>::fma(acc.b, a, b.b);
@@ -732,8 +737,11 @@ __device__ __forceinline__ void wide_loop_tiled(const SpmmArgs &a, const Cx &cx0
 // is register-allocated alone.  Epilogue: empty C rows are zeroed.
 // resident blocks per SM: wider J slices per lane (NV float4) need more
 // registers for the accumulators and the gathers in flight (no spills)
+#ifndef LF_V8_MIN_BLOCKS
+#define LF_V8_MIN_BLOCKS 3  // 8 floats per lane (80 registers)
+#endif
 constexpr int min_blocks(int NV, int VEC = 4) {
-    return NV * VEC >= 16 ? 2 : NV * VEC == 8 ? 3 : kMinBlocks;
+    return NV * VEC >= 16 ? 2 : NV * VEC == 8 ? LF_V8_MIN_BLOCKS : kMinBlocks;
 }
 
 template <int VEC, int G, int NV, bool FULL, bool MD = false>

@@ -145,6 +145,63 @@ float run_tma(const float4 *tab, const int *idx, int64_t n, float4 *out, int blo
   return ms / it;
 }
 
+// LDGSTS variant: every lane cp.async-copies its 16 B of each row into a
+// per-warp shared-memory ring (no registers held while in flight); rows are
+// committed in groups of 4 and read back by the same lane (LDS.128), so in-
+// flight depth is bounded by shared memory, not registers.  D rows in flight.
+template <int D, int WPB, bool CG>
+__global__ void __launch_bounds__(WPB * 32) replay_lds(const float4 *__restrict__ tab, const int *__restrict__ idx,
+                                                        int64_t n_idx, float4 *__restrict__ out) {
+  extern __shared__ __align__(128) float4 ring[];
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  float4 *my = ring + (size_t)w * D * 32;
+  const int64_t gw = (int64_t)blockIdx.x * WPB + w, nw = (int64_t)gridDim.x * WPB;
+  const int64_t per = ((n_idx + nw - 1) / nw + 3) & ~int64_t(3);
+  const int64_t q0 = gw * per, q1 = min(n_idx, q0 + per) & ~int64_t(3);
+  float4 acc = make_float4(0, 0, 0, 0);
+  constexpr int G = D / 4;  // groups of 4 rows in flight
+  auto issue4 = [&](int64_t q) {  // rows q..q+3 into slots (q - q0) % D
+    if (q < q1) {
+#pragma unroll
+      for (int u = 0; u < 4; u++) {
+        const int r = __ldg(idx + q + u);
+        const uint32_t d = (uint32_t)__cvta_generic_to_shared(my + (size_t)((q - q0 + u) % D) * 32 + lane);
+        const float4 *src = tab + (int64_t)r * 32 + lane;
+        if (CG) asm volatile("cp.async.cg.shared.global [%0], [%1], 16;" ::"r"(d), "l"(src) : "memory");
+        else asm volatile("cp.async.ca.shared.global [%0], [%1], 16;" ::"r"(d), "l"(src) : "memory");
+      }
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+  for (int g = 0; g < G; g++) issue4(q0 + 4 * g);
+  for (int64_t q = q0; q < q1; q += 4) {
+    asm volatile("cp.async.wait_group %0;" ::"n"(G - 1) : "memory");
+#pragma unroll
+    for (int u = 0; u < 4; u++) {
+      const float4 v = my[(size_t)((q - q0 + u) % D) * 32 + lane];
+      acc.x += v.x; acc.y += v.y; acc.z += v.z; acc.w += v.w;
+    }
+    issue4(q + 4 * G);
+  }
+  asm volatile("cp.async.wait_all;" ::: "memory");
+  if (acc.x + acc.y + acc.z + acc.w == 12345.f) out[0] = acc;
+}
+
+template <int D, int WPB, bool CG>
+float run_lds(const float4 *tab, const int *idx, int64_t n, float4 *out, int bps, int sms) {
+  const size_t smem = (size_t)WPB * D * 512;
+  CK(cudaFuncSetAttribute(replay_lds<D, WPB, CG>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem));
+  cudaEvent_t a, b; CK(cudaEventCreate(&a)); CK(cudaEventCreate(&b));
+  replay_lds<D, WPB, CG><<<sms * bps, WPB * 32, smem>>>(tab, idx, n, out);
+  CK(cudaGetLastError());
+  CK(cudaEventRecord(a));
+  const int it = 10;
+  for (int i = 0; i < it; i++) replay_lds<D, WPB, CG><<<sms * bps, WPB * 32, smem>>>(tab, idx, n, out);
+  CK(cudaEventRecord(b)); CK(cudaEventSynchronize(b));
+  float ms; CK(cudaEventElapsedTime(&ms, a, b));
+  return ms / it;
+}
+
 int main(int argc, char **argv) {
   if (argc < 4) { printf("usage: gather_replay cols.bin n_cols J\n"); return 1; }
   FILE *f = fopen(argv[1], "rb");
@@ -173,6 +230,14 @@ int main(int argc, char **argv) {
   for (int occ : {2, 4, 8})
     printf("{\"interleaved_blocks_per_sm\": %d, \"ms_u4\": %.4f, \"ms_u8\": %.4f}\n", occ,
            run<4, 0, 1>(tab, idx, n, J / 4, out, sms * occ), run<8, 0, 1>(tab, idx, n, J / 4, out, sms * occ));
+  if (getenv("LDS")) {
+    printf("{\"lds_d8_w8_b4_cg\": %.4f, \"lds_d16_w8_b2_cg\": %.4f, \"lds_d16_w8_b3_cg\": %.4f, \"lds_d32_w8_b1_cg\": %.4f, "
+           "\"lds_d16_w16_b1_cg\": %.4f, \"lds_d12_w8_b4_cg\": %.4f, \"lds_d16_w8_b3_ca\": %.4f, \"lds_d8_w16_b2_cg\": %.4f}\n",
+           run_lds<8, 8, true>(tab, idx, n, out, 4, sms), run_lds<16, 8, true>(tab, idx, n, out, 2, sms),
+           run_lds<16, 8, true>(tab, idx, n, out, 3, sms), run_lds<32, 8, true>(tab, idx, n, out, 1, sms),
+           run_lds<16, 16, true>(tab, idx, n, out, 1, sms), run_lds<12, 8, true>(tab, idx, n, out, 4, sms),
+           run_lds<16, 8, false>(tab, idx, n, out, 3, sms), run_lds<8, 16, true>(tab, idx, n, out, 2, sms));
+  }
   if (getenv("NO_TMA")) return 0;
   printf("{\"tma_r16_w8_b1\": %.4f, \"tma_r32_w4_b1\": %.4f, \"tma_r32_w6_b1\": %.4f, \"tma_r16_w4_b2\": %.4f, \"tma_r8_w8_b2\": %.4f}\n",
          run_tma<16, 8>(tab, idx, n, out, 1, sms), run_tma<32, 4>(tab, idx, n, out, 1, sms),
