@@ -155,11 +155,6 @@ template <> struct Vec<8> {
             : "l"(p));
         return v;
     }
-                : "=f"(v.a.x), "=f"(v.a.y), "=f"(v.a.z), "=f"(v.a.w), "=f"(v.b.x), "=f"(v.b.y), "=f"(v.b.z), "=f"(v.b.w)
-                : "l"(p));
-        return v;
-    }
-#endif
     static __device__ __forceinline__ void fma(T &acc, float a, const T &b) {
         Vec<4>::fma(acc.a, a, b.a);
         Vec<4>::fma(acc.b, a, b.b);
