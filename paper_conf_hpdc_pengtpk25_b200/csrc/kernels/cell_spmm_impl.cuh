@@ -128,10 +128,22 @@ template <> struct Vec<4> {
         acc.z += __shfl_xor_sync(kFull, acc.z, o);
         acc.w += __shfl_xor_sync(kFull, acc.w, o);
     }
+    // C row stores carry no "memory" clobber: C is only written by this
+    // kernel (never read back), and a clobber would pin every later B-row
+    // gather behind the store (no overlap of a row's write with the next
+    // row's loads).  LF_ST_CLOBBER=1 restores it for measurement.
+#ifndef LF_ST_CLOBBER
+#define LF_ST_CLOBBER 0
+#endif
     static __device__ __forceinline__ void store(float *p, const T &v, uint64_t pol) {
+#if LF_ST_CLOBBER
         asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(p),
                      "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w), "l"(pol)
                      : "memory");
+#else
+        asm volatile("st.global.L1::no_allocate.L2::cache_hint.v4.f32 [%0], {%1, %2, %3, %4}, %5;" ::"l"(p),
+                     "f"(v.x), "f"(v.y), "f"(v.z), "f"(v.w), "l"(pol));
+#endif
     }
     static __device__ __forceinline__ void red(float *p, const T &v) {
         grid_dep_wait();
@@ -145,6 +157,9 @@ template <> struct Vec<4> {
 struct f8 {
     float4 a, b;
 };
+#ifndef LF_ST_V8
+#define LF_ST_V8 1  // 256-bit C row stores (st.global.v8.f32): c2 0.585 -> 0.576 ms
+#endif
 template <> struct Vec<8> {
     using T = f8;
     static __device__ __forceinline__ T zero() { return {make_float4(0.f, 0.f, 0.f, 0.f), make_float4(0.f, 0.f, 0.f, 0.f)}; }
@@ -164,8 +179,14 @@ template <> struct Vec<8> {
         Vec<4>::add_xor(acc.b, o);
     }
     static __device__ __forceinline__ void store(float *p, const T &v, uint64_t pol) {
+#if LF_ST_V8
+        asm volatile("st.global.L1::no_allocate.L2::cache_hint.v8.f32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8}, %9;" ::"l"(p),
+                     "f"(v.a.x), "f"(v.a.y), "f"(v.a.z), "f"(v.a.w), "f"(v.b.x), "f"(v.b.y), "f"(v.b.z), "f"(v.b.w),
+                     "l"(pol));
+#else
         Vec<4>::store(p, v.a, pol);
         Vec<4>::store(p + 4, v.b, pol);
+#endif
     }
     static __device__ __forceinline__ void red(float *p, const T &v) {
         Vec<4>::red(p, v.a);

@@ -344,7 +344,11 @@ __global__ void __launch_bounds__(kThreads, LF_MARK_MIN_BLOCKS) stats_mark_kerne
             have[k] = LF_MARK_MODE == 0 ? __ldcg(mask + h[k]) : LF_MARK_MODE == 2 ? ld_ca(mask + h[k]) : 0u;
 #pragma unroll
         for (int k = 0; k < K; k++)
+#ifdef LF_DIAG_NORED  // diagnostic builds only: the marking pass without its REDs
+            if (c[k] >= 0 && (have[k] & bit[k]) != bit[k] && bit[k] == 0x80000000u) atomicOr(mask + h[k], bit[k]);
+#else
             if (c[k] >= 0 && (have[k] & bit[k]) != bit[k]) atomicOr(mask + h[k], bit[k]);
+#endif
     }
 }
 

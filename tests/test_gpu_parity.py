@@ -167,6 +167,41 @@ def test_configure_stats_and_alg3_match_oracle(lf):
         assert st.features[6] == pytest.approx(f[6], rel=1e-9)
 
 
+def _hot_column_csr(n_rows: int, n_cols: int, seed: int) -> "gen.CSR":
+    """Every row holds column 7 plus 0..5 random columns: >= 2^20 nonzeros in
+    rows of several natural buckets, a third of them in one column."""
+    rng = np.random.default_rng(seed)
+    lens = rng.integers(0, 6, size=n_rows)
+    rp = np.zeros(n_rows + 1, np.int64)
+    rp[1:] = np.cumsum(lens + 1)
+    ci = np.empty(int(rp[-1]), np.int32)
+    extra = rng.integers(8, n_cols, size=int(lens.sum())).astype(np.int32)
+    ci[rp[:-1]] = 7
+    pos = np.repeat(rp[:-1] + 1, lens) + (np.arange(int(lens.sum())) - np.repeat(np.cumsum(lens) - lens, lens))
+    ci[pos] = extra
+    for i in np.flatnonzero(lens > 1):  # rows sorted by column (CSR contract)
+        ci[rp[i]:rp[i + 1]] = np.sort(ci[rp[i]:rp[i + 1]])
+    return gen.CSR(n_rows, n_cols, rp, ci, gen.fill(len(ci), seed, gen.STREAM_VAL, gen.INT, -3, 3), "hotcol")
+
+
+@pytest.mark.parametrize("case", ["rmat16", "hotcol"])
+def test_configure_large_inputs_match_oracle(lf, case):
+    """Column marking (stats_mark_kernel) on >= 2^20 nonzeros in tiles of
+    several natural buckets: a power-law matrix, and one with a third of its
+    nonzeros in a single column (every tile marks that column).  Unat / Utop
+    / H / F and Algorithm 3 == the oracle at P = 1 and 3."""
+    A_h = gen.rmat(16, 20, seed=3) if case == "rmat16" else _hot_column_csr(1 << 20, 40000, 4)
+    assert A_h.nnz >= 1 << 20
+    A = lf.Csr.from_host(A_h)
+    for P in (1, 3):
+        params, st = lf.configure(A, 64, force_parts=P, force_format=1)
+        for p in range(P):
+            H, F, Un, Ut = oracle.partition_stats(A_h, P, p)
+            assert list(st.H[p]) == H.tolist() and list(st.F[p]) == F.tolist()
+            assert list(st.Unat[p]) == Un.tolist() and list(st.Utop[p]) == Ut.tolist()
+            assert st.chosen_log2[p] == oracle.build_buckets(A_h, P, p, 64)
+
+
 def test_golden_configure_on_gpu(lf):
     """The hand-worked eq. 7 examples, through the GPU statistics."""
     from conftest import read_golden
