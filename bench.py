@@ -45,7 +45,10 @@ def peaks():
 # (tools/gather_replay.cu, profiles/r1_gather_replay.md): pure 512-B B-row
 # gathers at the best depth (U = 8, 4 blocks/SM), CSR order
 GATHER_CEILING = {"c2_rmat20": (20649.0, "profiles/r1_gather_replay.md: c2 column sequence replayed as pure "
-                                         "512-B row gathers, U=8, 4 blocks/SM, 0.399 ms")}
+                                         "512-B row gathers, U=8, 4 blocks/SM, 0.399 ms"),
+                  # c4 at P = 8 gathers 1-KB rows from a ~30 MB partition slab of B (L2-resident)
+                  "c4_reddit": (19244.0, "profiles/r1_gather_roofline.md: random 1024-B row gathers from an "
+                                         "L2-resident 96 MB table, 8 blocks/SM")}
 
 
 def src_hash():
@@ -632,6 +635,8 @@ def time_workload(lf, lfd, torch, dist, name, J, args, world, rank, dev, ev, max
     out = {"workload": name, "J": J, "n_rows": A_h.n_rows, "nnz": A_h.nnz, "distinct_cols": U,
            "params": params.as_dict(), "spmm_path": path, "spmm_ms": sp_ms, "step_ms_serial": step_ms,
            "gflops": flops / (sp_ms * 1e-3) / 1e9, "step_gflops": flops / (step_ms * 1e-3) / 1e9}
+    if path == "cell_spmm_kernel":  # per-slot path: one B-row gather per nonzero binds it
+        out["gather"] = gather_roofline(name, A_h.nnz, J, world, sp_ms)
     hbm_peak, peak_kind = peaks()
     gbs = bytes_alg / world / (sp_ms * 1e-3) / 1e9
     traffic, traffic_src = ncu_traffic(name, J) if world == 1 else (None, "N > 1")
