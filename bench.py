@@ -47,8 +47,8 @@ def peaks():
 GATHER_CEILING = {"c2_rmat20": (20649.0, "profiles/r1_gather_replay.md: c2 column sequence replayed as pure "
                                          "512-B row gathers, U=8, 4 blocks/SM, 0.399 ms"),
                   # c4 at P = 8 gathers 1-KB rows from a ~30 MB partition slab of B (L2-resident)
-                  "c4_reddit": (19244.0, "profiles/r1_gather_roofline.md: random 1024-B row gathers from an "
-                                         "L2-resident 96 MB table, 8 blocks/SM")}
+                  "c4_reddit": (20109.0, "profiles/r1_gather_roofline.md (round-2 rows): random 1024-B row gathers "
+                                         "from an L2-resident 32 MB table (c4's partition slab is 29 MB), 8 blocks/SM")}
 
 
 def src_hash():
@@ -512,9 +512,30 @@ def main():
         x1.record(pipe.s_d2h)
         pipe.synchronize()
         e2e_ms = maxr(x0.elapsed_time(x1) / n_e2e)
+        # PCIe floor of that step: the same H2D and D2H bytes copied concurrently
+        # (full duplex) on the pipeline's streams with no compute in between
+        sl, nz = pipe.slots[0], int(h_ci.numel())
+        y0, y1 = ev(), ev()
+        torch.cuda.synchronize()
+        y0.record(pipe.s_h2d)
+        pipe.s_d2h.wait_event(y0)
+        for i in range(n_e2e):
+            with torch.cuda.stream(pipe.s_h2d):
+                sl["rp"].copy_(h_rp, non_blocking=True)
+                sl["ci"][:nz].copy_(h_ci, non_blocking=True)
+                sl["va"][:nz].copy_(h_va, non_blocking=True)
+                sl["B"].copy_(h_B, non_blocking=True)
+            with torch.cuda.stream(pipe.s_d2h):
+                h_Cs[i % 2].copy_(pipe.slots[1]["C"], non_blocking=True)
+        pipe.s_h2d.wait_stream(pipe.s_d2h)
+        y1.record(pipe.s_h2d)
+        torch.cuda.synchronize()
+        pcie_ms = maxr(y0.elapsed_time(y1) / n_e2e)
         e2e = {"value": flops / (e2e_ms * 1e-3) / 1e9, "unit": "GFLOP/s", "ms_per_step": e2e_ms,
                "api": "HostPipeline.submit (host CSR + B in, host C out; N > 1: each rank's row block)",
-               "h2d_bytes_per_step": int(h2d * world), "d2h_bytes_per_step": int(d2h * world)}
+               "h2d_bytes_per_step": int(h2d * world), "d2h_bytes_per_step": int(d2h * world),
+               "pcie_floor_ms": pcie_ms, "pcie_frac": pcie_ms / e2e_ms,
+               "pcie_floor_note": "the step's H2D + D2H bytes copied concurrently on the same streams, no compute"}
         del pipe
     del C_full, C_loc, lane_C, d_rp, d_ci, d_va, d_B, A
     torch.cuda.empty_cache()

@@ -69,7 +69,7 @@ int main() {
   CK(cudaMemset(tab, 0, max_bytes));
   std::vector<int> h(n_idx);
   printf("{\"sms\": %d}\n", sms);
-  for (int64_t mb : {4, 16, 48, 96, 256, 1024}) {
+  for (int64_t mb : {4, 16, 32, 48, 96, 256, 1024}) {
     for (int row_bytes : {512, 1024}) {
       const int64_t rows = mb * (1LL << 20) / row_bytes;
       uint64_t s = 88172645463325252ull;
