@@ -46,6 +46,10 @@ def peaks():
 # gathers at the best depth (U = 8, 4 blocks/SM), CSR order
 GATHER_CEILING = {"c2_rmat20": (20649.0, "profiles/r1_gather_replay.md: c2 column sequence replayed as pure "
                                          "512-B row gathers, U=8, 4 blocks/SM, 0.399 ms"),
+                  # permuted R-MAT: c2's column sequence replayed in shuffled order (the row
+                  # permutation's effect) ran at 0.403 ms = 20,437 GB/s
+                  "c2p_rmat20_perm": (20437.0, "profiles/r1_gather_replay.md: c2 column sequence replayed in "
+                                               "shuffled order, U=8, 4 blocks/SM, 0.403 ms"),
                   # c4 at P = 8 gathers 1-KB rows from a ~30 MB partition slab of B (L2-resident)
                   "c4_reddit": (20109.0, "profiles/r1_gather_roofline.md (round-2 rows): random 1024-B row gathers "
                                          "from an L2-resident 32 MB table (c4's partition slab is 29 MB), 8 blocks/SM")}
@@ -261,7 +265,7 @@ def run_reference(args):
 # --------------------------------------------------------------------------
 # GPU arm
 # --------------------------------------------------------------------------
-DEFAULT_EXTRA = "c3b_banded2M:128,c3b_banded2M:64,c3_stencil126:64,c3_stencil126:128,c4_reddit:256"
+DEFAULT_EXTRA = "c3b_banded2M:128,c3b_banded2M:64,c3_stencil126:64,c3_stencil126:128,c4_reddit:256,c2p_rmat20_perm:128"
 
 
 def maybe_spawn(args):

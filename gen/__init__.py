@@ -230,6 +230,7 @@ def random_small(n_rows: int, n_cols: int, max_len: int, seed: int, dup: bool = 
 CONFIGS = {
     "c1_uniform1024": dict(J=32),
     "c2_rmat20": dict(J=128),
+    "c2p_rmat20_perm": dict(J=128),
     "c3_stencil126": dict(J=64),
     # configs[2] read literally ("banded FEM-like 2M rows, ~50M nnz"): a band
     # of half-width 12 around the diagonal, 25 nonzeros per interior row
@@ -244,6 +245,10 @@ def config(name: str, seed: int = 0, kind: int = GRID, lo: int = -3, hi: int = 3
         m = uniform(1024, 1024, 1.0 / 64.0, seed, kind, lo, hi)
     elif name == "c2_rmat20":
         m = rmat(20, 16, seed=seed, kind=kind, lo=lo, hi=hi)
+    elif name == "c2p_rmat20_perm":
+        # the same R-MAT with rows and columns permuted ("also
+        # report a permuted variant"): hub rows / columns scattered over the index range
+        m = rmat(20, 16, seed=seed, permute=True, kind=kind, lo=lo, hi=hi)
     elif name == "c3_stencil126":
         m = stencil27(126, seed, kind, lo, hi)
     elif name == "c3b_banded2M":

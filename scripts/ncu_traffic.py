@@ -23,7 +23,7 @@ ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
 import bench  # noqa: E402
 
-DEFAULT = ["c2_rmat20:128", "c3b_banded2M:64", "c3b_banded2M:128", "c3_stencil126:64", "c3_stencil126:128",
+DEFAULT = ["c2_rmat20:128", "c2p_rmat20_perm:128", "c3b_banded2M:64", "c3b_banded2M:128", "c3_stencil126:64", "c3_stencil126:128",
            "c4_reddit:256"]
 KREGEX = "regex:cell_spmm|csr_spmm|zero_rows"
 
