@@ -201,11 +201,7 @@ __global__ void __launch_bounds__(kThreads, LF_MARK_MIN_BLOCKS) stats_mark_kerne
     __shared__ uint8_t rt0[kMarkTile + 1]; // t0 of the tile's rows (P == 1)
     __shared__ int32_t wsum[kThreads / 32];
     constexpr int kFB = LF_MARK_FBITS16 ? kMarkFilter / 2 : kMarkFilter;
-    __shared__ uint32_t fkey[kMarkFilter], fbits[kFB];  // block filter of uniform tiles
-    for (int q = threadIdx.x; q < kMarkFilter; q += blockDim.x) {
-        fkey[q] = kFilterEmpty;
-        if (q < kFB) fbits[q] = 0u;
-    }
+    __shared__ uint32_t fkey[kMarkFilter], fbits[kFB];  // block filter of uniform tiles (cleared below)
     constexpr int K = kMarkTile / kThreads;
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     __shared__ unsigned s_tmin, s_tmax;  // natural buckets of the tile's non-empty rows (P == 1)
@@ -258,6 +254,13 @@ __global__ void __launch_bounds__(kThreads, LF_MARK_MIN_BLOCKS) stats_mark_kerne
     // every non-empty row of the tile in one natural bucket (banded, stencil,
     // regular rows): every nonzero gets that bit, no position -> row scan
     const bool uni = P == 1 && s_tmin == s_tmax;
+    if (LF_MARK_MODE == 3 && (uni || LF_MARK_FILTER_ALL)) {  // only filtered tiles clear the filter
+        // (ordered before its use by the __syncthreads after the scan)
+        for (int q = threadIdx.x; q < kMarkFilter; q += blockDim.x) {
+            fkey[q] = kFilterEmpty;
+            if (q < kFB) fbits[q] = 0u;
+        }
+    }
     if (!uni) {  // inclusive scan of cnt, conflict-free: warp w scans its 512 entries in
        // 32-wide chunks (shuffles), then adds the totals of the warps before it
         constexpr int PER_WARP = kMarkTile / (kThreads / 32);
