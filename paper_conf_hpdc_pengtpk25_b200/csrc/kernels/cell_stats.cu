@@ -14,9 +14,11 @@
 //                       (column, bits) pairs in a shared-memory filter first
 //   stats_cols_kernel   one thread per mask slot: Unat[p][t] = #{c : bit t},
 //                       Utop[p][t] = #{c : highest bit >= t} (bit transpose)
-// and, for the grouped SpMM path's decision, group_sample_kernel (sampled
-// distinct columns of 4-row groups); features_kernel reads the row lengths
-// alone when the statistics pass is not run speculatively (lf_api.cu).
+// and, for the grouped / windowed SpMM paths' decision, the group samples
+// (group_sample_warp: distinct columns of 4-row groups, B-row windows of
+// 128-row groups), taken by extra blocks of stats_rows_kernel or, on the
+// features-first path, by group_sample_kernel; features_kernel reads the row
+// lengths alone when the statistics pass is not run speculatively (lf_api.cu).
 #include "../lf_internal.cuh"
 
 namespace lf {
@@ -77,6 +79,86 @@ __device__ __forceinline__ void block_len_stats(unsigned long long mn, unsigned 
     }
 }
 
+// Grouped-path heuristic (cell_spmm.cu "grouped path"): on kGroupSamples
+// groups of kGroupRows consecutive rows spread evenly over A (rows of at most
+// 32 nonzeros; a group with a longer row is skipped), the number of DISTINCT
+// columns of the group and its nonzeros, summed.  Their ratio says how many
+// B-row gathers merging the group's columns saves.  A warp per group, the
+// distinct columns counted in a per-warp shared-memory hash set.
+constexpr int kGroupSamples = 2048;
+__device__ __forceinline__ void group_sample_warp(const int64_t *__restrict__ row_ptr,
+                                                  const int32_t *__restrict__ col, int64_t n_rows, StatsDev *st,
+                                                  int64_t smp, int32_t *hs_w) {
+    const int lane = threadIdx.x & 31;
+    for (int q = lane; q < 256; q += 32) hs_w[q] = -1;
+    __syncwarp();
+    if (smp >= kGroupSamples) return;
+    // tcgen05 windowed path (cell_spmm_tc.cu): the B-row window of 128
+    // consecutive rows = [min first column, max last column]; rows longer than
+    // 32 make the sample ineligible (the path needs every W <= 32)
+    {
+        const int64_t n_wg = n_rows / 128;
+        if (n_wg > 0) {
+            const int64_t i0 = (smp * n_wg / kGroupSamples) * 128;
+            const int64_t base0 = row_ptr[0];
+            int mn = INT32_MAX, mx = -1;
+            bool ok = true;
+            for (int r = lane; r < 128; r += 32) {
+                const int64_t b = row_ptr[i0 + r] - base0, e = row_ptr[i0 + r + 1] - base0;
+                ok = ok && e - b <= 32;
+                if (e > b) {
+                    mn = min(mn, col[base0 + b]);
+                    mx = max(mx, col[base0 + e - 1]);
+                }
+            }
+            ok = __all_sync(kFull, ok);
+            mn = __reduce_min_sync(kFull, mn);
+            mx = __reduce_max_sync(kFull, mx);
+            if (lane == 0 && ok && mx >= 0) {
+                const unsigned long long span = (unsigned long long)(mx - mn + 1);
+                atomicAdd(&st->win_span, span);
+                atomicAdd(&st->win_cnt, 1ull);
+                if (span > 256) atomicAdd(&st->win_over, 1ull);
+            }
+        }
+    }
+    const int64_t n_groups = n_rows / kGroupRows;
+    if (n_groups == 0) return;
+    const int64_t i0 = (smp * n_groups / kGroupSamples) * kGroupRows;
+    const int64_t base = row_ptr[0];
+    int64_t b[kGroupRows], l[kGroupRows];
+    bool ok = true;
+#pragma unroll
+    for (int r = 0; r < kGroupRows; r++) {
+        b[r] = row_ptr[i0 + r] - base;
+        l[r] = row_ptr[i0 + r + 1] - base - b[r];
+        ok = ok && l[r] <= 32;
+    }
+    if (!ok) return;
+    const int32_t *colb = col + base;
+    unsigned n_u = 0, n_nz = 0;
+#pragma unroll
+    for (int r = 0; r < kGroupRows; r++) {
+        const int32_t c = lane < l[r] ? colb[b[r] + lane] : -1;
+        bool need = c >= 0, ins = false;
+        int h = (int)(((uint32_t)c * 0x9E3779B1u) >> 24);
+        while (__any_sync(kFull, need)) {
+            if (need) {
+                const int prev = atomicCAS(&hs_w[h], -1, c);
+                if (prev == -1) ins = true;
+                if (prev == -1 || prev == c) need = false;
+                else h = (h + 1) & 255;
+            }
+        }
+        n_u += __popc(__ballot_sync(kFull, ins));
+        n_nz += (unsigned)l[r];
+    }
+    if (lane == 0) {
+        atomicAdd(&st->grp_union, (unsigned long long)n_u);
+        atomicAdd(&st->grp_nnz, (unsigned long long)n_nz);
+    }
+}
+
 // Pass 1 -- one thread per row: segments of the row in every partition, their
 // natural bucket t0 (written to t0seg[i*P+p]), the H / F histograms
 // (warp-aggregated: __match_any_sync for H, REDUX for F) and the Table 2
@@ -94,14 +176,26 @@ __global__ void __launch_bounds__(kThreads) stats_rows_kernel(const int64_t *__r
                                                               int64_t S, int P, StatsDev *st,
                                                               uint8_t *__restrict__ t0seg,
                                                               int64_t *__restrict__ tile_row,
-                                                              int64_t *__restrict__ tile_pos) {
+                                                              int64_t *__restrict__ tile_pos, int rows_grid) {
+    if ((int)blockIdx.x >= rows_grid) {
+        // the blocks after the row blocks take the grouped / windowed path samples
+        // (group_sample_warp): independent of the row pass, so they run beside it
+        __shared__ int32_t hs[8][256];
+        const int w = threadIdx.x >> 5;
+        group_sample_warp(row_ptr, col, n_rows, st, (int64_t)(blockIdx.x - rows_grid) * 8 + w, hs[w]);
+        return;
+    }
     extern __shared__ unsigned long long sh[];  // H_s[P][32], F_s[P][32]
     unsigned long long *H_s = sh, *F_s = sh + P * kMaxT;
     for (int q = threadIdx.x; q < 2 * P * kMaxT; q += blockDim.x) sh[q] = 0;
     __syncthreads();
     const int lane = threadIdx.x & 31;
     unsigned long long mn = ~0ull, mx = 0, sum = 0, sq = 0;
-    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    // P = 1: lane t keeps H[t] / F[t] of its warp in registers (a 64-bit
+    // shared-memory atomicAdd is a CAS loop: per row batch it was a quarter
+    // of the kernel's instructions); added to the block's table once
+    unsigned long long accH = 0, accF = 0;
+    const int64_t stride = (int64_t)rows_grid * blockDim.x;
     for (int64_t base = (int64_t)blockIdx.x * blockDim.x; base < n_rows; base += stride) {
         const int64_t i = base + threadIdx.x;
         const bool active = i < n_rows;
@@ -130,19 +224,37 @@ __global__ void __launch_bounds__(kThreads) stats_rows_kernel(const int64_t *__r
             const int64_t l = e - b;
             const int t0 = l > 0 ? ceil_log2_i64(l) : kMaxT;
             if (active) t0seg[i * P + p] = l > 0 ? (uint8_t)t0 : kEmpty;
-            const unsigned peers = __match_any_sync(kFull, t0);
-            if (t0 < kMaxT && (peers & ((1u << lane) - 1u)) == 0)
-                atomicAdd(&H_s[p * kMaxT + t0], (unsigned long long)__popc(peers));
             const int tmax = __reduce_max_sync(kFull, l > 0 ? (unsigned)t0 : 0u);
-            if (__any_sync(kFull, l > 0)) {
-                for (int t = 0; t <= tmax; t++) {
-                    const unsigned v = (l > 0 && t <= t0) ? (unsigned)((l + (int64_t(1) << t) - 1) >> t) : 0u;
-                    const unsigned long long sv = warp_sum_u31(v);
-                    if (lane == 0 && sv) atomicAdd(&F_s[p * kMaxT + t], sv);
+            if (P == 1) {
+                if (__any_sync(kFull, l > 0)) {
+                    for (int t = 0; t <= tmax; t++) {
+                        const unsigned v = (l > 0 && t <= t0) ? (unsigned)((l + (int64_t(1) << t) - 1) >> t) : 0u;
+                        const unsigned long long sv = warp_sum_u31(v);
+                        const unsigned hc = __popc(__ballot_sync(kFull, l > 0 && t0 == t));
+                        if (lane == t) {
+                            accF += sv;
+                            accH += hc;
+                        }
+                    }
+                }
+            } else {
+                const unsigned peers = __match_any_sync(kFull, t0);
+                if (t0 < kMaxT && (peers & ((1u << lane) - 1u)) == 0)
+                    atomicAdd(&H_s[p * kMaxT + t0], (unsigned long long)__popc(peers));
+                if (__any_sync(kFull, l > 0)) {
+                    for (int t = 0; t <= tmax; t++) {
+                        const unsigned v = (l > 0 && t <= t0) ? (unsigned)((l + (int64_t(1) << t) - 1) >> t) : 0u;
+                        const unsigned long long sv = warp_sum_u31(v);
+                        if (lane == 0 && sv) atomicAdd(&F_s[p * kMaxT + t], sv);
+                    }
                 }
             }
             b = e;
         }
+    }
+    if (P == 1 && lane < kMaxT) {
+        if (accH) atomicAdd(&H_s[lane], accH);
+        if (accF) atomicAdd(&F_s[lane], accF);
     }
     block_len_stats(mn, mx, sum, sq, st);  // its __syncthreads also orders the H_s / F_s updates
     for (int q = threadIdx.x; q < P * kMaxT; q += blockDim.x) {
@@ -447,86 +559,12 @@ uint32_t mask_slots(int64_t n_cols) {
     return (uint32_t)m;
 }
 
-// Grouped-path heuristic (cell_spmm.cu "grouped path"): on kGroupSamples
-// groups of kGroupRows consecutive rows spread evenly over A (rows of at most
-// 32 nonzeros; a group with a longer row is skipped), the number of DISTINCT
-// columns of the group and its nonzeros, summed.  Their ratio says how many
-// B-row gathers merging the group's columns saves.  A warp per group, the
-// distinct columns counted in a per-warp shared-memory hash set.
-constexpr int kGroupSamples = 2048;
 __global__ void __launch_bounds__(256) group_sample_kernel(const int64_t *__restrict__ row_ptr,
                                                            const int32_t *__restrict__ col, int64_t n_rows,
                                                            StatsDev *st) {
     __shared__ int32_t hs[8][256];
-    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
-    for (int q = lane; q < 256; q += 32) hs[w][q] = -1;
-    __syncwarp();
-    const int64_t smp = (int64_t)blockIdx.x * 8 + w;
-    if (smp >= kGroupSamples) return;
-    // tcgen05 windowed path (cell_spmm_tc.cu): the B-row window of 128
-    // consecutive rows = [min first column, max last column]; rows longer than
-    // 32 make the sample ineligible (the path needs every W <= 32)
-    {
-        const int64_t n_wg = n_rows / 128;
-        if (n_wg > 0) {
-            const int64_t i0 = (smp * n_wg / kGroupSamples) * 128;
-            const int64_t base0 = row_ptr[0];
-            int mn = INT32_MAX, mx = -1;
-            bool ok = true;
-            for (int r = lane; r < 128; r += 32) {
-                const int64_t b = row_ptr[i0 + r] - base0, e = row_ptr[i0 + r + 1] - base0;
-                ok = ok && e - b <= 32;
-                if (e > b) {
-                    mn = min(mn, col[base0 + b]);
-                    mx = max(mx, col[base0 + e - 1]);
-                }
-            }
-            ok = __all_sync(kFull, ok);
-            mn = __reduce_min_sync(kFull, mn);
-            mx = __reduce_max_sync(kFull, mx);
-            if (lane == 0 && ok && mx >= 0) {
-                const unsigned long long span = (unsigned long long)(mx - mn + 1);
-                atomicAdd(&st->win_span, span);
-                atomicAdd(&st->win_cnt, 1ull);
-                if (span > 256) atomicAdd(&st->win_over, 1ull);
-            }
-        }
-    }
-    const int64_t n_groups = n_rows / kGroupRows;
-    if (n_groups == 0) return;
-    const int64_t i0 = (smp * n_groups / kGroupSamples) * kGroupRows;
-    const int64_t base = row_ptr[0];
-    int64_t b[kGroupRows], l[kGroupRows];
-    bool ok = true;
-#pragma unroll
-    for (int r = 0; r < kGroupRows; r++) {
-        b[r] = row_ptr[i0 + r] - base;
-        l[r] = row_ptr[i0 + r + 1] - base - b[r];
-        ok = ok && l[r] <= 32;
-    }
-    if (!ok) return;
-    const int32_t *colb = col + base;
-    unsigned n_u = 0, n_nz = 0;
-#pragma unroll
-    for (int r = 0; r < kGroupRows; r++) {
-        const int32_t c = lane < l[r] ? colb[b[r] + lane] : -1;
-        bool need = c >= 0, ins = false;
-        int h = (int)(((uint32_t)c * 0x9E3779B1u) >> 24);
-        while (__any_sync(kFull, need)) {
-            if (need) {
-                const int prev = atomicCAS(&hs[w][h], -1, c);
-                if (prev == -1) ins = true;
-                if (prev == -1 || prev == c) need = false;
-                else h = (h + 1) & 255;
-            }
-        }
-        n_u += __popc(__ballot_sync(kFull, ins));
-        n_nz += (unsigned)l[r];
-    }
-    if (lane == 0) {
-        atomicAdd(&st->grp_union, (unsigned long long)n_u);
-        atomicAdd(&st->grp_nnz, (unsigned long long)n_nz);
-    }
+    const int w = threadIdx.x >> 5;
+    group_sample_warp(row_ptr, col, n_rows, st, (int64_t)blockIdx.x * 8 + w, hs[w]);
 }
 
 namespace {
@@ -576,15 +614,14 @@ cudaError_t launch_stats(const lf_csr &A, int P, StatsDev *d_stats, uint32_t *d_
         if (tiles > 0x7fffffff) return cudaErrorInvalidValue;
         int64_t *tile_row = reinterpret_cast<int64_t *>(d_t0seg + (((size_t)A.n_rows * P + 15) & ~size_t(15)));
         int64_t *tile_pos = tile_row + tiles;
-        stats_rows_kernel<<<grid, kThreads, hist, s>>>(A.row_ptr, A.col_ind, A.n_rows, S, P, d_stats, d_t0seg,
-                                                        tile_row, tile_pos);
+        const bool smp = sample && A.n_rows >= kGroupRows && A.nnz > 0;
+        stats_rows_kernel<<<grid + (smp ? kGroupSamples / 8 : 0), kThreads, hist, s>>>(
+            A.row_ptr, A.col_ind, A.n_rows, S, P, d_stats, d_t0seg, tile_row, tile_pos, grid);
         if (A.nnz > 0)
             stats_mark_kernel<<<(unsigned)tiles, kThreads, 0, s>>>(A.row_ptr, A.col_ind, A.n_rows, S, P, d_t0seg,
                                                                     tile_row, tile_pos, tiles, d_colmask,
                                                                     mask_slots(A.n_cols) - 1);
     }
-    if (sample && A.n_rows >= kGroupRows && A.nnz > 0)
-        group_sample_kernel<<<kGroupSamples / 8, 256, 0, s>>>(A.row_ptr, A.col_ind, A.n_rows, d_stats);
     if (A.n_cols > 0) {
         const int64_t want = ((int64_t)mask_slots(A.n_cols) + kThreads - 1) / kThreads;
         const int grid = (int)std::min<int64_t>(want, (int64_t)num_sms() * 8);
