@@ -17,7 +17,7 @@
 // and, for the grouped / windowed SpMM paths' decision, the group samples
 // (group_sample_warp: distinct columns of 4-row groups, B-row windows of
 // 128-row groups), taken by extra blocks of stats_rows_kernel or, on the
-// features-first path, by group_sample_kernel; features_kernel reads the row
+// features-first path, of features_kernel; features_kernel reads the row
 // lengths alone when the statistics pass is not run speculatively (lf_api.cu).
 #include "../lf_internal.cuh"
 
@@ -559,13 +559,6 @@ uint32_t mask_slots(int64_t n_cols) {
     return (uint32_t)m;
 }
 
-__global__ void __launch_bounds__(256) group_sample_kernel(const int64_t *__restrict__ row_ptr,
-                                                           const int32_t *__restrict__ col, int64_t n_rows,
-                                                           StatsDev *st) {
-    __shared__ int32_t hs[8][256];
-    const int w = threadIdx.x >> 5;
-    group_sample_warp(row_ptr, col, n_rows, st, (int64_t)blockIdx.x * 8 + w, hs[w]);
-}
 
 namespace {
 
@@ -574,10 +567,17 @@ namespace {
 // (8 B per row).  One thread per row, warp then block reduction, one set of
 // 64-bit atomics per block.  (Used when the statistics pass is too long to
 // run speculatively for P = 1, see lf_cell_configure.)
-__global__ void __launch_bounds__(kThreads) features_kernel(const int64_t *__restrict__ row_ptr, int64_t n_rows,
-                                                            StatsDev *st) {
+__global__ void __launch_bounds__(kThreads) features_kernel(const int64_t *__restrict__ row_ptr,
+                                                            const int32_t *__restrict__ col, int64_t n_rows,
+                                                            StatsDev *st, int rows_grid) {
+    if ((int)blockIdx.x >= rows_grid) {  // extra blocks: the group / window samples (as stats_rows_kernel)
+        __shared__ int32_t hs[8][256];
+        const int w = threadIdx.x >> 5;
+        group_sample_warp(row_ptr, col, n_rows, st, (int64_t)(blockIdx.x - rows_grid) * 8 + w, hs[w]);
+        return;
+    }
     unsigned long long mn = ~0ull, mx = 0, sum = 0, sq = 0;
-    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    const int64_t stride = (int64_t)rows_grid * blockDim.x;
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n_rows; i += stride) {
         const unsigned long long len = (unsigned long long)(__ldg(row_ptr + i + 1) - __ldg(row_ptr + i));
         mn = min(mn, len);
@@ -594,9 +594,9 @@ cudaError_t launch_features(const lf_csr &A, StatsDev *d_stats, cudaStream_t s) 
     if (A.n_rows <= 0) return cudaSuccess;
     const int64_t want = (A.n_rows + kThreads - 1) / kThreads;
     const int grid = (int)std::min<int64_t>(want, (int64_t)num_sms() * 8);
-    features_kernel<<<grid, kThreads, 0, s>>>(A.row_ptr, A.n_rows, d_stats);
-    if (A.n_rows >= kGroupRows && A.nnz > 0)
-        group_sample_kernel<<<kGroupSamples / 8, 256, 0, s>>>(A.row_ptr, A.col_ind, A.n_rows, d_stats);
+    const bool smp = A.n_rows >= kGroupRows && A.nnz > 0;
+    features_kernel<<<grid + (smp ? kGroupSamples / 8 : 0), kThreads, 0, s>>>(A.row_ptr, A.col_ind, A.n_rows,
+                                                                             d_stats, grid);
     return cudaGetLastError();
 }
 
