@@ -265,7 +265,7 @@ def test_row_shard_view(lf):
 
 
 # ---- full-size BASELINE configs, the bench's launch configuration ----------
-FULL = ["c1_uniform1024", "c2_rmat20", "c3_stencil126", "c3b_banded2M"]
+FULL = ["c1_uniform1024", "c2_rmat20", "c2p_rmat20_perm", "c3_stencil126", "c3b_banded2M"]
 
 
 @pytest.mark.parametrize("name", FULL)
@@ -347,7 +347,7 @@ def test_reddit_shard_p8(lf):
     spmm_check(M, sub, B_h, exact=True, rows=rows)
 
 
-@pytest.mark.parametrize("name", ["c2_rmat20", "c3_stencil126", "c3b_banded2M"])
+@pytest.mark.parametrize("name", ["c2_rmat20", "c2p_rmat20_perm", "c3_stencil126", "c3b_banded2M"])
 def test_full_configure_matches_oracle(lf, name):
     """Full-size configure (nnz > 2^25 takes the features-first path on c3 /
     c3b) against the oracle at the P the predictor chose: every eq. 7 cost of
