@@ -559,14 +559,15 @@ def main():
     hbm_peak, peak_kind = peaks()
     P = params.n_parts
     # configure (lf_api.cu): nnz <= 2^25 -> the statistics pass for P = 1 first
-    # (stats_rows, stats_mark, group_sample, stats_cols) and again if the
-    # predictor picks P > 1; larger -> features_kernel + group_sample first,
-    # then the statistics pass when CELL is used.  build: bucket_kernel<0>,
-    # tile_scan, pad_init, bucket_kernel<1>, slot_fill, run_bounds (+ seg_kernel
-    # for P > 1).  SpMM: zero_rows_kernel + the SpMM kernel; CSR: csr_spmm_kernel.
+    # (stats_rows carrying the group / window samples, stats_mark, stats_cols)
+    # and again (3 kernels) if the predictor picks P > 1; larger ->
+    # features_kernel (with the samples) first, then the statistics pass when
+    # CELL is used.  build: bucket_kernel<0>, tile_scan, pad_init,
+    # bucket_kernel<1>, slot_fill, run_bounds (+ seg_kernel for P > 1).  SpMM:
+    # zero_rows_kernel + the SpMM kernel; CSR: csr_spmm_kernel.
     spec = args.parts != 0 or A_h.nnz <= (1 << 25)
-    cfg_launches = (4 + (4 if (params.n_parts != 1 and args.parts == 0 and params.use_cell) else 0)) if spec \
-        else (2 + (4 if params.use_cell else 0))
+    cfg_launches = (3 + (3 if (params.n_parts != 1 and args.parts == 0 and params.use_cell) else 0)) if spec \
+        else (1 + (3 if params.use_cell else 0))
     if params.use_cell:
         launches_per_step = cfg_launches + 6 + (1 if P > 1 else 0) + 2
     else:
