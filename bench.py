@@ -236,7 +236,9 @@ def run_reference(args):
     if rank != 0:
         return 0
     import oracle
-    cores = oracle.set_threads(0)
+    # rank 0 alone runs the oracle (the other ranks exit without work), so it
+    # takes every host core even under torchrun, which sets OMP_NUM_THREADS=1
+    cores = oracle.set_threads(os.cpu_count() or 1)
     A_h, J = gen.config(args.config, args.seed)
     B_h = gen.dense(A_h.n_cols, J, args.seed)
     per_step = max(0.2, min(5.0, 120.0 / (args.steps + args.warmup)))
