@@ -202,6 +202,27 @@ def test_configure_large_inputs_match_oracle(lf, case):
             assert st.chosen_log2[p] == oracle.build_buckets(A_h, P, p, 64)
 
 
+def test_configure_very_long_rows(lf):
+    """Natural buckets up to t = 22 (rows of 1 .. 2^21 + 3 nonzeros, one of them
+    2^21 + 3 long, plus empty rows): H / F / Unat / Utop per bucket (the P = 1
+    statistics pass keeps H[t], F[t] of bucket t in lane t) == the oracle."""
+    rng = np.random.default_rng(11)
+    lens = np.concatenate([[0, 1, 2, 3, 5, 33, 1000, (1 << 21) + 3, 0, 70000], rng.integers(0, 40, 3000)])
+    n_cols = 1 << 22
+    rows = [np.sort(rng.choice(n_cols, size=int(l), replace=False)).astype(np.int32) if l else np.zeros(0, np.int32)
+            for l in lens]
+    rp = np.zeros(len(lens) + 1, np.int64)
+    rp[1:] = np.cumsum(lens)
+    ci = np.concatenate(rows)
+    A_h = gen.CSR(len(lens), n_cols, rp, ci, gen.fill(len(ci), 11, gen.STREAM_VAL, gen.INT, -3, 3), "longrows")
+    A = lf.Csr.from_host(A_h)
+    params, st = lf.configure(A, 32, force_parts=1, force_format=1)
+    H, F, Un, Ut = oracle.partition_stats(A_h, 1, 0)
+    assert list(st.H[0]) == H.tolist() and list(st.F[0]) == F.tolist()
+    assert list(st.Unat[0]) == Un.tolist() and list(st.Utop[0]) == Ut.tolist()
+    assert st.max_log2[0] == 22 and st.chosen_log2[0] == oracle.build_buckets(A_h, 1, 0, 32)
+
+
 def test_golden_configure_on_gpu(lf):
     """The hand-worked eq. 7 examples, through the GPU statistics."""
     from conftest import read_golden
