@@ -18,6 +18,9 @@
  *     crosses the ABI.  Argument checks are done on the host before any
  *     device work.  On LF_ERR_CUDA, lf_last_error_detail() holds the CUDA
  *     error string (thread-local, valid until the next call on the thread).
+ *     A call that launches work first clears a non-sticky CUDA error left
+ *     pending by earlier runtime calls of the thread, so its status reflects
+ *     its own launches (a sticky error still fails its first launch).
  *   - Matrices: A is I x K sparse (CSR on input, CELL after build); B is a
  *     dense K x J fp32 row-major matrix with leading dimension ldb >= J
  *     (elements); C is dense I x J fp32 row-major with ldc >= J.
@@ -254,7 +257,12 @@ LF_API lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, co
  * synchronisation.  The handle's arrays are immutable: concurrent calls on
  * different streams (and host threads) with different C are safe -- the
  * work-queue counter slot a launch uses is fenced behind that slot's previous
- * launch when it ran on another stream.  B must not alias C. */
+ * launch when it ran on another stream.  B must not alias C.
+ * CUDA graphs: calls on the handle's build stream launch kernels only and can
+ * be captured into a graph (a replay reuses the counter slots of the capture;
+ * replays of one graph must not overlap).  Calls on other streams record and
+ * wait on events of the build stream, so capture them only with the build
+ * stream in the same capture. */
 LF_API lf_status lf_spmm(const lf_cell *h, const float *B, int64_t ldb, int32_t J, float *C, int64_t ldc,
                   lf_stream_t s);
 

@@ -181,6 +181,13 @@ lf::SpmmArgs spmm_args(const lf_cell *h, const float *B, int64_t ldb, int32_t J,
 
 }  // namespace
 
+// Entry of every call that launches work: a non-sticky CUDA error left
+// pending by earlier, unrelated runtime calls of the process (cudaGetLastError
+// reports the LAST error of the thread) is cleared here, so the status of
+// this call reflects its own launches only.  A sticky error (a faulted
+// context) is not cleared by this and fails the call's first launch.
+static void clear_stale_error() { (void)cudaGetLastError(); }
+
 extern "C" {
 
 int32_t lf_abi_version(void) { return LF_ABI_VERSION; }
@@ -203,6 +210,7 @@ const char *lf_last_error_detail(void) { return g_detail.c_str(); }
 lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts *opts, lf_cell_params *out,
                             lf_configure_stats *stats, lf_stream_t stream) {
     g_detail.clear();
+    clear_stale_error();
     if (lf_status st = check_csr(A)) return st;
     if (!out) return fail(LF_ERR_INVALID_ARG, "out is NULL");
     if (J < 1) return fail(LF_ERR_INVALID_ARG, "J < 1");
@@ -377,6 +385,7 @@ lf_status lf_cell_configure(const lf_csr *A, int32_t J, const lf_configure_opts 
 lf_status lf_cell_build(const lf_csr *A, const lf_cell_params *params, const lf_configure_stats *stats,
                         const lf_allocator *al, lf_stream_t stream, lf_cell **out) {
     g_detail.clear();
+    clear_stale_error();
     if (lf_status st = check_csr(A)) return st;
     if (!params || !out) return fail(LF_ERR_INVALID_ARG, "params/out is NULL");
     *out = nullptr;
@@ -664,6 +673,7 @@ lf_status lf_spmm(const lf_cell *h, const float *B, int64_t ldb, int32_t J, floa
 lf_status lf_spmm_ex(const lf_cell *h, const float *B, int64_t ldb, int32_t J, float *C, int64_t ldc,
                      const lf_spmm_opts *opts, lf_stream_t stream) {
     g_detail.clear();
+    clear_stale_error();
     if (!h) return fail(LF_ERR_INVALID_ARG, "handle is NULL");
     if (J < 0 || ldb < J || ldc < J || ldb < 0 || ldc < 0) return fail(LF_ERR_INVALID_ARG, "need 0 <= J <= ldb, ldc");
     const int n_dst = opts ? opts->n_dst : 0;
@@ -743,6 +753,7 @@ const char *lf_spmm_kernel_name(const lf_cell *h, int32_t J) {
 lf_status lf_csr_spmm(const lf_csr *A, const float *B, int64_t ldb, int32_t J, float *C, int64_t ldc,
                       lf_stream_t stream) {
     g_detail.clear();
+    clear_stale_error();
     if (lf_status st = check_csr(A)) return st;
     if (J < 0 || ldb < J || ldc < J) return fail(LF_ERR_INVALID_ARG, "need 0 <= J <= ldb, ldc");
     if (J == 0 || A->n_rows == 0) return LF_OK;

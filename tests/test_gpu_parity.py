@@ -571,3 +571,34 @@ def test_kernel_name(lf):
     assert lf.CellMatrix.build(R, p, s).path(128) == "cell_spmm_kernel"
     p, s = lf.configure(R, 128, force_format=2)
     assert lf.CellMatrix.build(R, p, s).path(128) == "csr_spmm_kernel"
+
+
+def test_spmm_in_cuda_graph(lf):
+    """lf_spmm on the handle's build stream launches kernels only, so it can be
+    captured in a CUDA graph: 8 captured launches (more than one counter
+    slot each replay), replayed 3 times, give Alg. 1's C each time; the
+    fixed-CSR kernel too."""
+    A_h = gen.rmat(12, 16, seed=21, kind=gen.INT)
+    A = lf.Csr.from_host(A_h)
+    J = 64
+    B_h = gen.dense(A_h.n_cols, J, 21, gen.INT, -15, 15)
+    B = torch.from_numpy(B_h).cuda()
+    Cref = oracle.spmm_csr(A_h, B_h)[0]
+    for fmt in (1, 2):
+        s = torch.cuda.Stream()
+        params, stats = lf.configure(A, J, force_format=fmt, stream=s)
+        M = lf.CellMatrix.build(A, params, stats, stream=s)
+        C = torch.empty((A_h.n_rows, J), device="cuda")
+        with torch.cuda.stream(s):
+            M.spmm(B, out=C, stream=s)  # warm (not captured)
+        s.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=s):
+            for _ in range(8):
+                M.spmm(B, out=C, stream=torch.cuda.current_stream())
+        for _ in range(3):
+            C.fill_(float("nan"))
+            g.replay()
+            torch.cuda.synchronize()
+            assert np.array_equal(C.cpu().numpy().astype(np.float64), Cref), M.path()
+        M.close()
